@@ -1,0 +1,410 @@
+// ga_bench.cu -- workload kernels behind include/ga_bench.h.
+//
+// Trace kernels run the same request trace through ga_malloc/ga_free or
+// through CUDA's built-in device malloc/free (the paper's baseline).
+// Correctness mode: one kernel per phase, allocation log + lifetime tags.
+// Timing mode: one persistent kernel, nothing but allocator calls.
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <cstdio>
+
+#include "ga.h"
+#include "ga_bench.h"
+#include "ga_device.cuh"
+#include "ga_internal.h"
+
+namespace {
+
+constexpr uint64_t kNullOff = ~0ull;
+
+struct GaPolicy {
+    ga_dev_heap h;
+    __device__ void* alloc(uint64_t n) const { return ga_malloc(h, n); }
+    __device__ void release(void* p) const { ga_free(h, p); }
+    __device__ uint64_t off(const void* p) const { return p ? (uint64_t)((const char*)p - h.base) : kNullOff; }
+    __device__ void* ptr(uint64_t o) const { return o == kNullOff ? nullptr : (void*)(h.base + o); }
+};
+struct CudaPolicy {
+    __device__ void* alloc(uint64_t n) const { return malloc(n); }
+    __device__ void release(void* p) const { free(p); }
+    __device__ uint64_t off(const void* p) const { return p ? (uint64_t)p : kNullOff; }
+    __device__ void* ptr(uint64_t o) const { return o == kNullOff ? nullptr : (void*)o; }
+};
+
+__device__ __forceinline__ uint64_t tag_of(uint32_t t, uint32_t r) { return 0xA5A5000000000000ull | ((uint64_t)r << 24) | t; }
+__device__ __forceinline__ void tag_write(void* p, uint32_t n, uint64_t tag) {
+    char* b = (char*)p;
+    *(volatile uint64_t*)b = tag;
+    *(volatile uint64_t*)(b + ((n - 8) & ~7u)) = tag ^ 0xFFull;
+}
+__device__ __forceinline__ bool tag_ok(const void* p, uint32_t n, uint64_t tag) {
+    const char* b = (const char*)p;
+    return *(const volatile uint64_t*)b == tag && *(const volatile uint64_t*)(b + ((n - 8) & ~7u)) == (tag ^ 0xFFull);
+}
+__device__ __forceinline__ void logw(ga_log_rec* log, uint64_t idx, uint64_t off, uint32_t size, uint32_t meta) {
+    if (!log) return;
+    ga_log_rec r; r.off = off; r.size = size; r.meta = meta;
+    log[idx] = r;
+}
+__device__ __forceinline__ uint32_t meta_of(uint32_t t, uint32_t r, uint32_t op) { return t | (r << 20) | (op << 31); }
+
+// warp-aggregated counter flush
+__device__ __forceinline__ void flush_counts(uint64_t* counts, uint32_t nm, uint32_t nf, uint32_t nfree, uint32_t nbad) {
+    unsigned act = __activemask();
+    uint32_t a = __reduce_add_sync(act, nm), b = __reduce_add_sync(act, nf), c = __reduce_add_sync(act, nfree),
+             d = __reduce_add_sync(act, nbad);
+    if ((int)(threadIdx.x & 31) == __ffs(act) - 1) {
+        if (a) atomicAdd((unsigned long long*)&counts[0], a);
+        if (b) atomicAdd((unsigned long long*)&counts[1], b);
+        if (c) atomicAdd((unsigned long long*)&counts[2], c);
+        if (d) atomicAdd((unsigned long long*)&counts[3], d);
+    }
+}
+
+// D == 1 correctness round r in [0, R]: free the held block, then malloc (r < R)
+template <class P>
+__global__ void __launch_bounds__(256) k_churn_round(P al, const uint32_t* sizes, uint32_t R, uint32_t T, uint32_t r,
+                                                     uint64_t* held, ga_log_rec* log, uint64_t* counts, uint32_t flags) {
+    uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= T) return;
+    uint32_t nm = 0, nf = 0, nfree = 0, nbad = 0;
+    uint64_t idx = 2ull * ((uint64_t)r * T + t);
+    uint64_t hp = held[2 * t];
+    uint32_t hs = (uint32_t)held[2 * t + 1];
+    if (hp != kNullOff) {
+        void* p = al.ptr(hp);
+        if ((flags & GA_TRACE_TAG) && !tag_ok(p, hs, tag_of(t, r - 1))) nbad++;
+        al.release(p);
+        nfree++;
+        logw(log, idx + 1, hp, hs, meta_of(t, r, 1));
+    } else logw(log, idx + 1, kNullOff, 0, 0);
+    hp = kNullOff; hs = 0;
+    uint32_t n = r < R ? sizes[(uint64_t)r * T + t] : 0;
+    if (n) {
+        void* p = al.alloc(n);
+        nm++;
+        if (!p) nf++;
+        else {
+            if (flags & GA_TRACE_TAG) tag_write(p, n, tag_of(t, r));
+            hp = al.off(p); hs = n;
+        }
+        logw(log, idx, al.off(p), n, meta_of(t, r, 0));
+    } else logw(log, idx, kNullOff, 0, 0);
+    held[2 * t] = hp;
+    held[2 * t + 1] = hs;
+    flush_counts(counts, nm, nf, nfree, nbad);
+}
+
+// D == 0 correctness: phase 0 mallocs every round-r block, phase 1 frees them
+template <class P>
+__global__ void __launch_bounds__(256) k_phase(P al, const uint32_t* sizes, uint32_t T, uint32_t r, uint32_t phase,
+                                               uint64_t* held, ga_log_rec* log, uint64_t* counts, uint32_t flags) {
+    uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= T) return;
+    uint32_t nm = 0, nf = 0, nfree = 0, nbad = 0;
+    uint64_t idx = 2ull * ((uint64_t)r * T + t);
+    if (phase == 0) {
+        uint32_t n = sizes[(uint64_t)r * T + t];
+        uint64_t hp = kNullOff;
+        if (n) {
+            void* p = al.alloc(n);
+            nm++;
+            if (!p) nf++;
+            else { if (flags & GA_TRACE_TAG) tag_write(p, n, tag_of(t, r)); hp = al.off(p); }
+            logw(log, idx, al.off(p), n, meta_of(t, r, 0));
+        } else logw(log, idx, kNullOff, 0, 0);
+        held[2 * t] = hp;
+        held[2 * t + 1] = hp == kNullOff ? 0 : n;
+    } else {
+        uint64_t hp = held[2 * t];
+        uint32_t hs = (uint32_t)held[2 * t + 1];
+        if (hp != kNullOff) {
+            void* p = al.ptr(hp);
+            if ((flags & GA_TRACE_TAG) && !tag_ok(p, hs, tag_of(t, r))) nbad++;
+            al.release(p);
+            nfree++;
+            logw(log, idx + 1, hp, hs, meta_of(t, r, 1));
+        } else logw(log, idx + 1, kNullOff, 0, 0);
+        held[2 * t] = kNullOff;
+        held[2 * t + 1] = 0;
+    }
+    flush_counts(counts, nm, nf, nfree, nbad);
+}
+
+// timing mode: every round in one kernel
+template <class P>
+__global__ void __launch_bounds__(256) k_timed(P al, const uint32_t* __restrict__ sizes, uint32_t R, uint32_t T, uint32_t D,
+                                               uint64_t* counts) {
+    uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= T) return;
+    uint32_t nm = 0, nf = 0, nfree = 0;
+    void* held = nullptr;
+    for (uint32_t r = 0; r < R; r++) {
+        uint32_t n = __ldg(&sizes[(uint64_t)r * T + t]);
+        if (D) {
+            if (held) { al.release(held); nfree++; held = nullptr; }
+            if (n) { held = al.alloc(n); nm++; nf += held == nullptr; }
+        } else if (n) {
+            void* p = al.alloc(n);
+            nm++;
+            if (p) { al.release(p); nfree++; } else nf++;
+        }
+    }
+    if (held) { al.release(held); nfree++; }
+    flush_counts(counts, nm, nf, nfree, 0);
+}
+
+// --------------------------------------------------------------------------
+// L2-atomic peak microbenchmark
+// --------------------------------------------------------------------------
+__global__ void k_l2_atomic(int pattern, uint64_t* buf, uint64_t n_words, uint32_t iters, uint64_t* sink, uint32_t zero) {
+    uint64_t tid = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    uint64_t acc = 0;
+    uint64_t* w;
+    switch (pattern) {
+        case 0: case 1: case 4: w = buf + (tid * 4) % n_words; break;
+        case 2: w = buf + (tid & zero); break;                     // runtime-uniform, not provably
+        case 3: w = buf + (tid % 1184) * 4; break;
+        default: { uint32_t sm; asm volatile("mov.u32 %0, %%smid;" : "=r"(sm)); w = buf + (uint64_t)(sm % 148) * 4; }
+    }
+    if (pattern == 1) {
+        for (uint32_t i = 0; i < iters; i++) atomicAdd((unsigned long long*)w, 1ull + (tid & zero));
+    } else if (pattern == 4 || pattern == 5) {
+        for (uint32_t i = 0; i < iters; i++) {
+            unsigned long long old = *(volatile unsigned long long*)w, prev;
+            while ((prev = atomicCAS((unsigned long long*)w, old, old + 1)) != old) old = prev;
+            acc += old;
+        }
+    } else {
+        for (uint32_t i = 0; i < iters; i++) acc += atomicAdd((unsigned long long*)w, 1ull + (tid & zero));
+    }
+    if (acc == 0x123456789ull) sink[0] = acc;                     // keep the returns live
+}
+
+// --------------------------------------------------------------------------
+// bulk-semaphore microbenchmark (Sec. 5.1)
+// --------------------------------------------------------------------------
+__device__ __forceinline__ uint32_t rnd_k(uint64_t seed, uint64_t tid, uint32_t it) {
+    uint64_t z = seed ^ (tid * 0x9E3779B97F4A7C15ull) ^ ((uint64_t)it * 0xBF58476D1CE4E5B9ull);
+    z += 0x9E3779B97F4A7C15ull;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    z ^= z >> 31;
+    return 1 + (uint32_t)(z % 32);
+}
+
+__global__ void k_bsem(ga_bsem_cfg cfg, uint64_t* sems, uint64_t* out, uint32_t zero) {
+    uint64_t tid = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    uint32_t sm; asm volatile("mov.u32 %0, %%smid;" : "=r"(sm));
+    uint32_t si = cfg.n_sems > 1 ? sm % cfg.n_sems : 0;
+    uint64_t* s = sems + (uint64_t)si * 4 + (tid & zero);
+    uint64_t* bump = sems + (uint64_t)cfg.n_sems * 4;             // the "resource": one atomic per batch
+    uint64_t granted = 0, waits = 0, batches = 0, produced = 0;
+    for (uint32_t it = 0; it < cfg.iters; it++) {
+        uint32_t k = cfg.k ? cfg.k : rnd_k(cfg.seed, tid, it);
+        if (cfg.variant == 2) k = 1;
+        if (cfg.variant == 0) {
+            unsigned act = __activemask();
+            unsigned grp = __match_any_sync(act, si);
+            uint32_t N = __reduce_add_sync(grp, k);
+            if ((int)(threadIdx.x & 31) == __ffs(grp) - 1) {
+                uint32_t Bp = cfg.B * ((N + cfg.B - 1) / cfg.B);
+                int r = ga_bsem_wait((ga_bsem*)s, N, Bp);
+                waits++;
+                if (r == GA_GROW) {
+                    atomicAdd((unsigned long long*)bump, (unsigned long long)Bp);
+                    batches += Bp / cfg.B; produced += Bp;
+                    ga_bsem_signal((ga_bsem*)s, Bp - N, Bp - N);
+                }
+                granted += N;
+                if (!cfg.acquire_only) ga_bsem_signal((ga_bsem*)s, N, 0);
+            }
+            __syncwarp(act);
+        } else if (cfg.variant == 1) {
+            uint32_t Bp = cfg.B * ((k + cfg.B - 1) / cfg.B);
+            int r = ga_bsem_wait((ga_bsem*)s, k, Bp);
+            waits++;
+            if (r == GA_GROW) {
+                atomicAdd((unsigned long long*)bump + (tid & zero), (unsigned long long)Bp);
+                batches += Bp / cfg.B; produced += Bp;
+                ga_bsem_signal((ga_bsem*)s, Bp - k, Bp - k);
+            }
+            granted += k;
+            if (!cfg.acquire_only) ga_bsem_signal((ga_bsem*)s, k, 0);
+        } else if (cfg.variant == 2) {
+            // growable counting semaphore (Sec. 3.2): S in the low 32 bits
+            int* S = (int*)s;
+            for (;;) {
+                int v = *(volatile int*)S;
+                if (v >= 1) { if (atomicCAS(S, v, v - 1) == v) break; continue; }
+                if (v == 0) {
+                    if (atomicCAS(S, 0, -1) == 0) {            // we grow: produce B, keep 1
+                        atomicAdd((unsigned long long*)bump + (tid & zero), (unsigned long long)cfg.B);
+                        batches++; produced += cfg.B;
+                        __threadfence();
+                        atomicAdd(S, (int)cfg.B);             // -1 + B: B - 1 left for others
+                        break;
+                    }
+                    continue;
+                }
+                __nanosleep(64);                               // blocked while S < 0
+            }
+            waits++;
+            granted += 1;
+            if (!cfg.acquire_only) atomicAdd(S, 1);
+        } else {
+            unsigned long long* c = (unsigned long long*)s;
+            atomicAdd(c, (unsigned long long)(-(long long)k) + (tid & zero));
+            waits++;
+            granted += k;
+            if (!cfg.acquire_only) atomicAdd(c, (unsigned long long)k + (tid & zero));
+        }
+    }
+    unsigned act = __activemask();
+    uint64_t g = granted, w = waits, b = batches, p = produced;
+    for (int o = 16; o; o >>= 1) {
+        g += __shfl_down_sync(act, g, o); w += __shfl_down_sync(act, w, o);
+        b += __shfl_down_sync(act, b, o); p += __shfl_down_sync(act, p, o);
+    }
+    if ((threadIdx.x & 31) == 0) {
+        atomicAdd((unsigned long long*)&out[0], g); atomicAdd((unsigned long long*)&out[1], w);
+        atomicAdd((unsigned long long*)&out[2], b); atomicAdd((unsigned long long*)&out[3], p);
+    }
+}
+__global__ void k_bsem_final(uint32_t n_sems, const uint64_t* sems, uint64_t* out, uint32_t variant) {
+    if (threadIdx.x || blockIdx.x) return;
+    int64_t sc = 0, md = 0;
+    for (uint32_t i = 0; i < n_sems; i++) {
+        uint64_t w = sems[i * 4];
+        int64_t C, D;
+        if (variant <= 1) { C = (int32_t)(uint32_t)(w >> 32); D = (int32_t)((uint32_t)w - 0x80000000u); }
+        else if (variant == 2) { C = (int32_t)(uint32_t)w; D = 0; }
+        else { C = (int64_t)w; D = 0; }
+        sc += C;
+        if ((D < 0 ? -D : D) > md) md = D < 0 ? -D : D;
+    }
+    out[4] = (uint64_t)sc; out[5] = (uint64_t)md;
+}
+__global__ void k_bsem_init(uint32_t n_sems, uint64_t* sems, uint32_t variant) {
+    uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < n_sems * 4 + 4) sems[i] = (variant <= 1 && i < n_sems * 4) ? 0x80000000ull : 0ull;
+}
+
+inline uint32_t nblocks(uint32_t T, uint32_t block) { return (T + block - 1) / block; }
+inline ga_status launched() { return cudaGetLastError() == cudaSuccess ? GA_OK : GA_ECUDA; }
+
+}  // namespace
+
+extern "C" {
+
+ga_status ga_trace_phase(ga_heap_t h, ga_stream_t stream, const uint32_t* sizes, uint32_t R, uint32_t T, uint32_t D,
+                         uint32_t round, uint32_t phase, uint64_t* held, ga_log_rec* log, uint64_t* counts,
+                         uint32_t flags, uint32_t block) {
+    if (!h || !sizes || !held || !counts || T == 0 || D > 1) return GA_EINVAL;
+    if (block == 0) block = 256;
+    GaPolicy al{h->dev};
+    cudaStream_t s = (cudaStream_t)stream;
+    if (!(flags & GA_TRACE_LOG)) log = nullptr;
+    if (D == 1) {
+        if (round > R) return GA_EINVAL;
+        k_churn_round<GaPolicy><<<nblocks(T, block), block, 0, s>>>(al, sizes, R, T, round, held, log, counts, flags);
+    } else {
+        if (round >= R || phase > 1) return GA_EINVAL;
+        k_phase<GaPolicy><<<nblocks(T, block), block, 0, s>>>(al, sizes, T, round, phase, held, log, counts, flags);
+    }
+    return launched();
+}
+
+ga_status ga_trace_timed(ga_heap_t h, ga_stream_t stream, const uint32_t* sizes, uint32_t R, uint32_t T, uint32_t D,
+                         uint64_t* counts, uint32_t block) {
+    if (!h || !sizes || !counts || T == 0 || D > 1) return GA_EINVAL;
+    if (block == 0) block = 256;
+    GaPolicy al{h->dev};
+    k_timed<GaPolicy><<<nblocks(T, block), block, 0, (cudaStream_t)stream>>>(al, sizes, R, T, D, counts);
+    return launched();
+}
+
+ga_status ga_trace_timed_host(ga_heap_t h, ga_stream_t stream, const uint32_t* host_sizes, uint32_t R, uint32_t T,
+                              uint32_t D, uint64_t* host_counts, uint32_t block) {
+    if (!h || !host_sizes || !host_counts || T == 0 || D > 1) return GA_EINVAL;
+    cudaStream_t s = (cudaStream_t)stream;
+    size_t sz = (size_t)R * T * 4;
+    size_t need = sz + 256 + 64;
+    if (h->scratch_bytes < need) {
+        if (h->scratch) cudaFree(h->scratch);
+        h->scratch = nullptr; h->scratch_bytes = 0;
+        if (cudaMalloc(&h->scratch, need) != cudaSuccess) return GA_ENOMEM;
+        h->scratch_bytes = need;
+    }
+    uint32_t* d_sizes = (uint32_t*)h->scratch;
+    uint64_t* d_counts = (uint64_t*)((char*)h->scratch + ((sz + 255) / 256) * 256);
+    if (cudaMemsetAsync(d_counts, 0, 64, s) != cudaSuccess) return GA_ECUDA;
+    if (cudaMemcpyAsync(d_sizes, host_sizes, sz, cudaMemcpyHostToDevice, s) != cudaSuccess) return GA_ECUDA;
+    ga_status st = ga_trace_timed(h, stream, d_sizes, R, T, D, d_counts, block);
+    if (st != GA_OK) return st;
+    if (cudaMemcpyAsync(host_counts, d_counts, 32, cudaMemcpyDeviceToHost, s) != cudaSuccess) return GA_ECUDA;
+    return cudaStreamSynchronize(s) == cudaSuccess ? GA_OK : GA_ECUDA;
+}
+
+ga_status ga_cuda_set_heap_limit(size_t bytes) {
+    return cudaDeviceSetLimit(cudaLimitMallocHeapSize, bytes) == cudaSuccess ? GA_OK : GA_ECUDA;
+}
+
+ga_status ga_cuda_trace_phase(ga_stream_t stream, const uint32_t* sizes, uint32_t R, uint32_t T, uint32_t D,
+                              uint32_t round, uint32_t phase, uint64_t* held, uint64_t* counts, uint32_t flags,
+                              uint32_t block) {
+    if (!sizes || !held || !counts || T == 0 || D > 1) return GA_EINVAL;
+    if (block == 0) block = 256;
+    CudaPolicy al;
+    cudaStream_t s = (cudaStream_t)stream;
+    if (D == 1) {
+        if (round > R) return GA_EINVAL;
+        k_churn_round<CudaPolicy><<<nblocks(T, block), block, 0, s>>>(al, sizes, R, T, round, held, nullptr, counts, flags);
+    } else {
+        if (round >= R || phase > 1) return GA_EINVAL;
+        k_phase<CudaPolicy><<<nblocks(T, block), block, 0, s>>>(al, sizes, T, round, phase, held, nullptr, counts, flags);
+    }
+    return launched();
+}
+
+ga_status ga_cuda_trace_timed(ga_stream_t stream, const uint32_t* sizes, uint32_t R, uint32_t T, uint32_t D,
+                              uint64_t* counts, uint32_t block) {
+    if (!sizes || !counts || T == 0 || D > 1) return GA_EINVAL;
+    if (block == 0) block = 256;
+    k_timed<CudaPolicy><<<nblocks(T, block), block, 0, (cudaStream_t)stream>>>(CudaPolicy{}, sizes, R, T, D, counts);
+    return launched();
+}
+
+ga_status ga_kernel_info(int which, uint32_t block, int* regs, int* blocks_per_sm, int* local_bytes) {
+    if (block == 0) block = 256;
+    cudaFuncAttributes a;
+    const void* f = which == 0 ? (const void*)k_timed<GaPolicy> : which == 1 ? (const void*)k_churn_round<GaPolicy>
+                                                                              : (const void*)k_timed<CudaPolicy>;
+    if (cudaFuncGetAttributes(&a, f) != cudaSuccess) return GA_ECUDA;
+    int nb = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, f, (int)block, 0) != cudaSuccess) return GA_ECUDA;
+    if (regs) *regs = a.numRegs;
+    if (blocks_per_sm) *blocks_per_sm = nb;
+    if (local_bytes) *local_bytes = (int)a.localSizeBytes;
+    return GA_OK;
+}
+
+ga_status ga_l2_atomic_bench(ga_stream_t stream, int pattern, uint64_t* d_buf, uint64_t n_words, uint32_t iters,
+                             uint32_t grid, uint32_t block, uint64_t* d_sink) {
+    if (!d_buf || !d_sink || pattern < 0 || pattern > 5 || n_words < 1184 * 4) return GA_EINVAL;
+    k_l2_atomic<<<grid, block, 0, (cudaStream_t)stream>>>(pattern, d_buf, n_words, iters, d_sink, 0u);
+    return launched();
+}
+
+ga_status ga_bsem_bench(ga_stream_t stream, const ga_bsem_cfg* cfg, uint64_t* sems, uint64_t* out) {
+    if (!cfg || !sems || !out || cfg->variant > 3 || cfg->B == 0 || cfg->n_sems == 0 || cfg->k > 32) return GA_EINVAL;
+    cudaStream_t s = (cudaStream_t)stream;
+    k_bsem_init<<<(cfg->n_sems * 4 + 4 + 255) / 256, 256, 0, s>>>(cfg->n_sems, sems, cfg->variant);
+    cudaMemsetAsync(out, 0, 64, s);
+    k_bsem<<<cfg->grid, cfg->block, 0, s>>>(*cfg, sems, out, 0u);
+    k_bsem_final<<<1, 32, 0, s>>>(cfg->n_sems, sems, out, cfg->variant);
+    return launched();
+}
+
+}  // extern "C"
