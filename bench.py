@@ -1,0 +1,351 @@
+#!/usr/bin/env python
+"""Benchmark: malloc+free calls/s of the B200-native allocator vs CUDA device malloc.
+
+Contract (driver): ``python bench.py --gpus N --steps K --warmup W`` prints ONE JSON
+line on rank 0.  One "step" = one pass of the whole hot path over one batch: the
+mixed-size churn trace d4 (BASELINE.json configs[3]) at full B200
+occupancy -- 303,104 threads x 16 rounds of {free previous block; malloc 16 B..64 KiB}
+plus the final free-all, on a 4 GiB heap ("pressure": ~71 % of the heap live after
+rounding) -- run as ONE kernel (timing mode, ga_trace_timed).  ``value`` = malloc
+calls (failed ones included) + frees, per second, summed over ranks.
+
+N > 1: one process per GPU, each with its own heap (replicas, no data-path
+collective); timing is the max over ranks.
+
+``--impl reference``: the reference arm is the sequential CPU oracle (oracle/),
+timed on this host on the same trace (rank 0 only).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import tracegen  # noqa: E402
+
+METRIC = "malloc+free calls/s on 1 B200 vs CUDA device malloc; fragmentation ratio"
+UNIT = "calls/s"
+L2_FLUSH_BYTES = 512 << 20
+
+
+# ----------------------------------------------------------------------------- helpers
+def algorithmic_atomics(sizes: np.ndarray) -> int:
+    """Minimum L2 atomics the method must issue for one pass of a D=1 trace with
+    every call succeeding: per warp-round and size class,
+    a group of N lanes needs 1 semaphore op + ceil(N / slots-per-bitmap-word)
+    tracking ops (bins: min(64, 4096/class); tree: 64 nodes per level word), for
+    the mallocs and again for the frees of the same blocks."""
+    R, T = sizes.shape
+    n = sizes.astype(np.int64)
+    lg = np.ceil(np.log2(np.maximum(n, 16))).astype(np.int64)           # class log2
+    key = lg - 4                                                        # 0..7 bins, 8.. tree
+    W = T // 32
+    k = key[:, : W * 32].reshape(R, W, 32)
+    total = 0
+    for c in range(int(key.max()) + 1):
+        N = (k == c).sum(axis=2)
+        per_word = min(64, 4096 >> (c + 4)) if c < 8 else 64
+        total += int(((N > 0) * (1 + (N + per_word - 1) // per_word)).sum())
+    return 2 * total
+
+
+class Clocks:
+    """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
+
+    def __init__(self, index: int):
+        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+             "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", "-i", str(index), f"--query-gpu={q}",
+                                       "--format=csv,noheader,nounits", "-lms", "100"],
+                                      stdout=self.f, stderr=subprocess.DEVNULL)
+        except OSError:
+            self.p = None
+
+    def stop(self) -> dict:
+        if self.p is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.p.terminate()
+        self.p.wait()
+        self.f.seek(0)
+        rows = [r.split(", ") for r in self.f.read().strip().splitlines() if r.strip()]
+        os.unlink(self.f.name)
+        sm = [float(r[1]) for r in rows if len(r) >= 9 and r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in rows if len(r) >= 9 and r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in rows if len(r) >= 9 for i in range(4) if r[5 + i].strip() == "Active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(rows)}
+
+
+def cpu_cores() -> int:
+    return len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else os.cpu_count()
+
+
+def oracle_leg(trace, budget_s: float = 10.0) -> dict:
+    """The oracle as it stands, on this host, 1 thread: the whole trace, repeated
+    until ~budget_s of CPU work (bounded sample)."""
+    import oracle
+    oracle.build()
+    runs, calls, t_total, st = 0, 0, 0.0, None
+    while t_total < budget_s or runs == 0:
+        t0 = time.perf_counter()
+        r = oracle.run_trace(trace.sizes, trace.heap_bytes, trace.D, want_ok=False)
+        t_total += time.perf_counter() - t0
+        st = r.stats
+        calls += st["calls"]
+        runs += 1
+        if runs >= 64:
+            break
+    return {"value": calls / t_total, "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": f"{trace.name}: whole trace ({trace.R} rounds x {trace.T} threads, "
+                      f"{st['calls']} calls) x {runs} runs, sequential C oracle, {t_total:.1f} s",
+            "seconds": t_total, "stats": st}
+
+
+# ----------------------------------------------------------------------------- reference arm
+def run_reference(args, trace):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    import oracle
+    oracle.build()
+    for _ in range(args.warmup):
+        oracle.run_trace(trace.sizes, trace.heap_bytes, trace.D, want_ok=False)
+    times, calls = [], 0
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        r = oracle.run_trace(trace.sizes, trace.heap_bytes, trace.D, want_ok=False)
+        times.append(time.perf_counter() - t0)
+        calls = r.stats["calls"]
+    ms = 1e3 * sum(times) / len(times)
+    value = calls / (ms / 1e3)
+    out = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+           "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+           "scaling": "weak", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
+           "config": config_of(trace, args),
+           "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle",
+                            "sample": f"{trace.name}: the whole trace per step ({calls} calls), sequential C oracle"},
+           "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+           "fragmentation": {"oracle": r.stats["peak_reserved_bytes"] / max(1, r.stats["peak_live_bytes"])}}
+    print(json.dumps(out), flush=True)
+    return 0
+
+
+def config_of(trace, args):
+    return {"workload": trace.name, "threads": trace.T, "rounds": trace.R, "free_depth": trace.D,
+            "heap_bytes": trace.heap_bytes, "sizes": "n = 2^k + U[1,2^k], k~U{3..15} (16 B - 64 KiB classes)",
+            "block": args.block, "l2": "flushed between steps (512 MiB write)", "seed": hex(trace.seed)}
+
+
+# ----------------------------------------------------------------------------- our arm
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--block", type=int, default=256)
+    ap.add_argument("--no-extras", action="store_true", help="skip CUDA-malloc, sweep, frag, cpu legs")
+    ap.add_argument("--cuda-budget-s", type=float, default=20.0)
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+
+    trace = tracegen.d4_mixed("pressure")
+    if args.impl == "reference":
+        return run_reference(args, trace)
+
+    import torch
+    import paper_conf_ppopp_geladog19_b200 as ga
+    from paper_conf_ppopp_geladog19_b200.runner import GpuHeap, run_correctness
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local)
+    stream = torch.cuda.current_stream(dev)
+
+    # per-rank trace (replicas: seed + rank); rank 0 uses the canonical trace
+    if rank:
+        trace = tracegen.Trace(trace.name, tracegen.mixed_sizes(trace.seed + rank, trace.R, trace.T), trace.D,
+                               trace.heap_bytes, trace.seed + rank)
+    R, T, D = trace.R, trace.T, trace.D
+    if not args.no_extras:
+        ga.ga_cuda_set_heap_limit(trace.heap_bytes)       # before any kernel that uses malloc
+    heap = GpuHeap(trace.heap_bytes, device=local, stream=stream)
+    d_sizes = torch.from_numpy(trace.sizes.view(np.int32)).to(dev)
+    counts = torch.zeros(8, dtype=torch.int64, device=dev)
+    flush = torch.empty(L2_FLUSH_BYTES // 4, dtype=torch.int32, device=dev)
+
+    def step():
+        ga.ga_trace_timed(heap.h, stream.cuda_stream, d_sizes.data_ptr(), R, T, D, counts.data_ptr(), args.block)
+
+    for _ in range(args.warmup):
+        flush.fill_(1)
+        step()
+    torch.cuda.synchronize()
+    counts.zero_()
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    clocks = Clocks(local)
+    if dist:
+        dist.barrier()
+    torch.cuda.synchronize()
+    t_wall = time.perf_counter()
+    for s, e in ev:
+        flush.fill_(s.__hash__() & 7)                      # L2 flush, outside the events
+        s.record(stream)
+        step()
+        e.record(stream)
+    torch.cuda.synchronize()
+    if dist:
+        dist.barrier()
+    wall = time.perf_counter() - t_wall
+    clk = clocks.stop()
+    kern_ms = [s.elapsed_time(e) for s, e in ev]
+    ms = sum(kern_ms) / len(kern_ms)
+    c = counts.cpu().numpy()
+    calls_step = int(c[0] + c[2]) // args.steps
+    fails_step = int(c[1]) // args.steps
+    t_max = torch.tensor([ms], device=dev, dtype=torch.float64)
+    tot_calls = torch.tensor([calls_step], device=dev, dtype=torch.float64)
+    if dist:
+        dist.all_reduce(t_max, op=dist.ReduceOp.MAX)
+        dist.all_reduce(tot_calls, op=dist.ReduceOp.SUM)
+    ms_max = float(t_max.item())
+    value = float(tot_calls.item()) / (ms_max / 1e3)
+
+    # ---- e2e: host buffers through the C ABI (H2D of the trace, kernel, D2H of counts)
+    h_sizes = torch.from_numpy(trace.sizes.view(np.int32)).pin_memory()
+    h_counts = np.zeros(4, dtype=np.uint64)
+    from paper_conf_ppopp_geladog19_b200.runner import run_timed_host
+    e2e_ms = []
+    for i in range(args.warmup + args.steps):
+        flush.fill_(2)
+        s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        s0.record(stream)
+        run_timed_host(heap, h_sizes, R, T, D, h_counts, args.block, stream)
+        s1.record(stream)
+        s1.synchronize()
+        if i >= args.warmup:
+            e2e_ms.append(s0.elapsed_time(s1))
+    e2e_calls = int(h_counts[0] + h_counts[2])
+    e2e_t = torch.tensor([sum(e2e_ms) / len(e2e_ms)], device=dev, dtype=torch.float64)
+    e2e_c = torch.tensor([e2e_calls], device=dev, dtype=torch.float64)
+    if dist:
+        dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
+        dist.all_reduce(e2e_c, op=dist.ReduceOp.SUM)
+    e2e = {"value": float(e2e_c.item()) / (float(e2e_t.item()) / 1e3), "unit": UNIT,
+           "h2d_bytes_per_step": int(trace.sizes.nbytes), "d2h_bytes_per_step": 32,
+           "ms_per_step": float(e2e_t.item())}
+
+    if rank != 0:
+        if dist:
+            dist.barrier()
+            dist.destroy_process_group()
+        return 0
+
+    # ---- roofline: L2 atomics, peak from the committed microbenchmark, measured live
+    buf = torch.zeros(148 * 8 * 256 * 4 + 8192, dtype=torch.int64, device=dev)
+    sink = torch.zeros(8, dtype=torch.int64, device=dev)
+    peaks = {}
+    grid, blk, iters = 148 * 8, 256, 64
+    for pat in (0, 1, 3):
+        for rep in range(3):
+            a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a0.record(stream)
+            ga.ga_l2_atomic_bench(stream.cuda_stream, pat, buf.data_ptr(), buf.numel(), iters, grid, blk,
+                                  sink.data_ptr())
+            a1.record(stream)
+            a1.synchronize()
+            if rep:
+                rate = grid * blk * iters / (a0.elapsed_time(a1) / 1e3) / 1e9
+                peaks[pat] = max(peaks.get(pat, 0.0), rate)
+    p_atom = max(peaks[0], peaks[1])
+    a_min = algorithmic_atomics(trace.sizes)
+    achieved = a_min / (ms / 1e3) / 1e9
+    kinfo = ga.ga_kernel_info(0, args.block)
+    roofline = {"bound": "l2_atomic", "achieved": achieved, "peak": p_atom, "unit": "Gatom/s",
+                "frac": achieved / p_atom, "traffic": None,
+                "per_launch_algorithmic_atomics": a_min,
+                "peak_source": "measured live: ga_l2_atomic_bench distinct-word ATOMG/REDG (max)",
+                "peak_patterns_gatom_s": {"atomg_distinct": peaks[0], "redg_distinct": peaks[1],
+                                          "atomg_1184_words": peaks[3]},
+                "kernel": {"regs": kinfo["regs"], "blocks_per_sm": kinfo["blocks_per_sm"],
+                           "stack_bytes": kinfo["local_bytes"]}}
+
+    out = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+           "warmup": args.warmup, "ms_per_step": ms_max, "higher_is_better": True, "scaling": "weak",
+           "vs_baseline": None, "dtype": "u64", "data": "synthetic",
+           "config": config_of(trace, args), "e2e": e2e, "gpu_launches": args.steps,
+           "clocks": clk, "roofline": roofline,
+           "calls_per_step": calls_step, "failed_mallocs_per_step": fails_step,
+           "kernel_ms": {"min": min(kern_ms), "max": max(kern_ms)}, "wall_s_timed_region": wall}
+
+    if not args.no_extras:
+        # ---- fragmentation (correctness mode: one kernel per round, reserved at boundaries)
+        heap.reset()
+        run = run_correctness(heap, trace.sizes, D, log=False, tag=False, reserved=True)
+        live_peak = run.peak_live_bytes                    # the GPU's own successful requests
+        cpu = oracle_leg(trace, budget_s=10.0)
+        frag_ora = cpu["stats"]["peak_reserved_bytes"] / cpu["stats"]["peak_live_bytes"]
+        frag_gpu = run.peak_reserved_bytes / live_peak if live_peak else None
+        out["fragmentation"] = {"gpu": frag_gpu, "oracle": frag_ora,
+                                "ratio": frag_gpu / frag_ora if frag_gpu else None,
+                                "gpu_peak_reserved_bytes": run.peak_reserved_bytes,
+                                "peak_live_bytes": live_peak,
+                                "oracle_peak_reserved_bytes": cpu["stats"]["peak_reserved_bytes"],
+                                "gpu_failed_mallocs": run.counts["n_fail"]}
+        cpu.pop("stats")
+        cpu.pop("seconds")
+        out["cpu_baseline"] = cpu
+
+        # ---- CUDA device malloc on the same trace (bounded prefix of rounds)
+        heap.reset()
+        torch.cuda.synchronize()
+        cc = torch.zeros(8, dtype=torch.int64, device=dev)
+        rr, t_cuda = 1, None
+        while True:
+            cc.zero_()
+            a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a0.record(stream)
+            ga.ga_cuda_trace_timed(stream.cuda_stream, d_sizes.data_ptr(), rr, T, D, cc.data_ptr(), args.block)
+            a1.record(stream)
+            a1.synchronize()
+            t_cuda = a0.elapsed_time(a1) / 1e3
+            if t_cuda * 2 > args.cuda_budget_s or rr >= R:
+                break
+            rr = min(R, rr * 2)
+        ccn = cc.cpu().numpy()
+        cuda_rate = float(ccn[0] + ccn[2]) / t_cuda
+        out["cuda_malloc"] = {"value": cuda_rate, "unit": UNIT, "rounds": rr,
+                              "failed_mallocs": int(ccn[1]), "seconds": t_cuda,
+                              "heap_limit_bytes": trace.heap_bytes}
+        out["speedup_vs_cuda_malloc"] = value / cuda_rate
+
+    print(json.dumps(out), flush=True)
+    if dist:
+        dist.barrier()
+        dist.destroy_process_group()
+    heap.close()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -33,14 +33,16 @@ struct CudaPolicy {
 };
 
 __device__ __forceinline__ uint64_t tag_of(uint32_t t, uint32_t r) { return 0xA5A5000000000000ull | ((uint64_t)r << 24) | t; }
+// tags: 8 bytes at the start and (n >= 16) 8 bytes at the last aligned slot of the request
 __device__ __forceinline__ void tag_write(void* p, uint32_t n, uint64_t tag) {
     char* b = (char*)p;
     *(volatile uint64_t*)b = tag;
-    *(volatile uint64_t*)(b + ((n - 8) & ~7u)) = tag ^ 0xFFull;
+    if (n >= 16) *(volatile uint64_t*)(b + ((n - 8) & ~7u)) = tag ^ 0xFFull;
 }
 __device__ __forceinline__ bool tag_ok(const void* p, uint32_t n, uint64_t tag) {
     const char* b = (const char*)p;
-    return *(const volatile uint64_t*)b == tag && *(const volatile uint64_t*)(b + ((n - 8) & ~7u)) == (tag ^ 0xFFull);
+    if (*(const volatile uint64_t*)b != tag) return false;
+    return n < 16 || *(const volatile uint64_t*)(b + ((n - 8) & ~7u)) == (tag ^ 0xFFull);
 }
 __device__ __forceinline__ void logw(ga_log_rec* log, uint64_t idx, uint64_t off, uint32_t size, uint32_t meta) {
     if (!log) return;

@@ -63,6 +63,11 @@ class TraceRun:
     log: np.ndarray | None = None
     peak_reserved_bytes: int = 0
     reserved_per_round: list = field(default_factory=list)
+    live_per_round: list = field(default_factory=list)   # requested bytes held at each boundary
+
+    @property
+    def peak_live_bytes(self) -> int:
+        return max(self.live_per_round) if self.live_per_round else 0
 
 
 def _counts(t: torch.Tensor) -> dict:
@@ -97,8 +102,8 @@ def run_correctness(heap: GpuHeap | None, sizes: np.ndarray, D: int, log: bool =
                 ga_cuda_trace_phase(s, d_sizes.data_ptr(), R, T, 1, r, 0, held.data_ptr(), counts.data_ptr(),
                                     flags, block)
             if heap and reserved and r < R:
-                rb = heap.reserved_bytes()
-                run.reserved_per_round.append(rb)
+                run.reserved_per_round.append(heap.reserved_bytes())
+                run.live_per_round.append(int(held[1::2].sum().item()))
         else:
             for ph in (0, 1):
                 if heap:
@@ -109,6 +114,7 @@ def run_correctness(heap: GpuHeap | None, sizes: np.ndarray, D: int, log: bool =
                                         flags, block)
                 if heap and reserved and ph == 0:
                     run.reserved_per_round.append(heap.reserved_bytes())
+                    run.live_per_round.append(int(held[1::2].sum().item()))
     st.synchronize()
     run.counts = _counts(counts)
     run.peak_reserved_bytes = max(run.reserved_per_round) if run.reserved_per_round else 0
