@@ -43,9 +43,9 @@ typedef struct {
     uint32_t bitmap_bits;   /* 256: out-of-band bitmap bits per page                   */
 } ga_layout_t;
 
-/* Plain-old-data view of a heap, passed BY VALUE to kernels that call
- * ga_malloc / ga_free.  Fields are owned by the library; do not modify. */
-typedef struct {
+/* Device-resident heap descriptor (lives at the start of the metadata
+ * allocation; device code reads it through L1).  Owned by the library. */
+typedef struct ga_desc {
     char* base;               /* pool base, 2 MiB aligned (R-31)                        */
     uint64_t pages;           /* usable pages (pool rounded down to whole chunks, R-30) */
     uint64_t nchunks;
@@ -70,6 +70,13 @@ typedef struct {
     uint64_t lvl_off[48];     /* word offset of level n (bits, then summaries)          */
     uint32_t lvl_words[48];   /* words of level n's bitmap                              */
     uint32_t lvl_sum1[48];    /* words of level n's first summary                       */
+} ga_desc;
+
+/* Plain-old-data handle passed BY VALUE to kernels that call ga_malloc /
+ * ga_free (16 bytes: cheap to pass, no per-thread copy of the descriptor). */
+typedef struct {
+    const ga_desc* desc;      /* device pointer to the descriptor                      */
+    char* base;               /* pool base (== desc->base)                             */
 } ga_dev_heap;
 
 typedef struct {

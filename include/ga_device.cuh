@@ -1,8 +1,8 @@
 /*
  * ga_device.cuh -- device interface of the B200-native throughput-oriented allocator.
  *
- *   __device__ void* ga_malloc(const ga_dev_heap& h, size_t n);
- *   __device__ void  ga_free  (const ga_dev_heap& h, void* p);
+ *   __device__ void* ga_malloc(ga_dev_heap h, size_t n);
+ *   __device__ void  ga_free  (ga_dev_heap h, void* p);
  *
  * The standard malloc / free interface for device threads (Gelado & Garland,
  * PPoPP'19), callable concurrently by every thread of a
@@ -31,13 +31,13 @@
 #include "ga.h"
 #include "../paper_conf_ppopp_geladog19_b200/csrc/ga_device_impl.cuh"
 
-__device__ __forceinline__ void* ga_malloc(const ga_dev_heap& h, size_t n) {
-    uint64_t off = ga::ga_malloc_off(h, (uint64_t)n);
+__device__ __forceinline__ void* ga_malloc(ga_dev_heap h, size_t n) {
+    uint64_t off = ga::ga_malloc_off(h.desc, (uint64_t)n);
     return off == ga::kNull ? nullptr : (void*)(h.base + off);
 }
 
-__device__ __forceinline__ void ga_free(const ga_dev_heap& h, void* p) {
-    ga::ga_free_off(h, p ? (uint64_t)((char*)p - h.base) : ga::kNull);
+__device__ __forceinline__ void ga_free(ga_dev_heap h, void* p) {
+    ga::ga_free_off(h.desc, p ? (uint64_t)((char*)p - h.base) : ga::kNull);
 }
 
 /* Bulk-semaphore primitives (Alg. 1 / Alg. 2), exported for the

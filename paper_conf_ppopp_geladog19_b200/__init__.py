@@ -48,14 +48,8 @@ class Stats(ctypes.Structure):
 
 
 class DevHeap(ctypes.Structure):
-    _fields_ = ([("base", ctypes.c_void_p), ("pages", ctypes.c_uint64), ("nchunks", ctypes.c_uint64),
-                 ("L", ctypes.c_uint32), ("n_arenas", ctypes.c_uint32), ("chunk_words", ctypes.c_uint32),
-                 ("flags", ctypes.c_uint32)] +
-                [(n, ctypes.c_void_p) for n in ("bits", "kind", "chunk_used", "chunk_owner", "chunk_nonfull",
-                                                "chunk_cand", "sem", "psem", "hint", "owned", "cand_any",
-                                                "avail", "tsem", "stats")] +
-                [("lvl_off", ctypes.c_uint64 * 48), ("lvl_words", ctypes.c_uint32 * 48),
-                 ("lvl_sum1", ctypes.c_uint32 * 48)])
+    """ga_dev_heap: the 16-byte handle kernels receive by value."""
+    _fields_ = [("desc", ctypes.c_void_p), ("base", ctypes.c_void_p)]
 
 
 class BsemCfg(ctypes.Structure):

@@ -19,7 +19,7 @@ namespace {
 constexpr uint64_t kNullOff = ~0ull;
 
 struct GaPolicy {
-    ga_dev_heap h;
+    ga_dev_heap h;      // 16-byte handle: descriptor pointer + base
     __device__ void* alloc(uint64_t n) const { return ga_malloc(h, n); }
     __device__ void release(void* p) const { ga_free(h, p); }
     __device__ uint64_t off(const void* p) const { return p ? (uint64_t)((const char*)p - h.base) : kNullOff; }
@@ -305,7 +305,7 @@ ga_status ga_trace_phase(ga_heap_t h, ga_stream_t stream, const uint32_t* sizes,
                          uint32_t flags, uint32_t block) {
     if (!h || !sizes || !held || !counts || T == 0 || D > 1) return GA_EINVAL;
     if (block == 0) block = 256;
-    GaPolicy al{h->dev};
+    GaPolicy al{ga_dev_heap{h->ddesc, h->dev.base}};
     cudaStream_t s = (cudaStream_t)stream;
     if (!(flags & GA_TRACE_LOG)) log = nullptr;
     if (D == 1) {
@@ -322,7 +322,7 @@ ga_status ga_trace_timed(ga_heap_t h, ga_stream_t stream, const uint32_t* sizes,
                          uint64_t* counts, uint32_t block) {
     if (!h || !sizes || !counts || T == 0 || D > 1) return GA_EINVAL;
     if (block == 0) block = 256;
-    GaPolicy al{h->dev};
+    GaPolicy al{ga_dev_heap{h->ddesc, h->dev.base}};
     k_timed<GaPolicy><<<nblocks(T, block), block, 0, (cudaStream_t)stream>>>(al, sizes, R, T, D, counts);
     return launched();
 }

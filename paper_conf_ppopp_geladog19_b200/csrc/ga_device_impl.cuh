@@ -81,7 +81,7 @@ static __device__ __forceinline__ void red_add_release(uint64_t* p, uint64_t v) 
     asm volatile("red.release.gpu.global.add.u64 [%0], %1;" :: "l"(p), "l"(v) : "memory");
 }
 static __device__ __forceinline__ void fence() { __threadfence(); }
-static __device__ __forceinline__ void stat_add(const ga_dev_heap& h, int i, uint64_t v) { a_add(&h.stats[i], v); }
+static __device__ __forceinline__ void stat_add(const ga_desc* h, int i, uint64_t v) { a_add(&h->stats[i], v); }
 
 static __device__ __forceinline__ uint32_t hash32(uint32_t x) {
     x ^= x >> 16; x *= 0x7feb352dU; x ^= x >> 15; x *= 0x846ca68bU; x ^= x >> 16; return x;
@@ -114,11 +114,11 @@ static __device__ __forceinline__ uint64_t valid_mask(int c, int w) {
     int s = (int)slots_of(c) - 64 * w;
     return s >= 64 ? ~0ull : s <= 0 ? 0ull : ((1ull << s) - 1);
 }
-static __device__ __forceinline__ uint32_t arena_of(const ga_dev_heap& h) { return smid() % h.n_arenas; }
-static __device__ __forceinline__ uint64_t* sem_ptr(const ga_dev_heap& h, uint32_t A, int c) { return h.sem + ((uint64_t)A * kNcls + c) * kSemStride; }
-static __device__ __forceinline__ uint64_t* psem_ptr(const ga_dev_heap& h, uint32_t A) { return h.psem + (uint64_t)A * kSemStride; }
-static __device__ __forceinline__ uint64_t* tsem_ptr(const ga_dev_heap& h, int n) { return h.tsem + (uint64_t)n * kSemStride; }
-static __device__ __forceinline__ uint64_t* page_bits(const ga_dev_heap& h, uint64_t p) { return h.bits + p * kBinWords; }
+static __device__ __forceinline__ uint32_t arena_of(const ga_desc* h) { return smid() % h->n_arenas; }
+static __device__ __forceinline__ uint64_t* sem_ptr(const ga_desc* h, uint32_t A, int c) { return h->sem + ((uint64_t)A * kNcls + c) * kSemStride; }
+static __device__ __forceinline__ uint64_t* psem_ptr(const ga_desc* h, uint32_t A) { return h->psem + (uint64_t)A * kSemStride; }
+static __device__ __forceinline__ uint64_t* tsem_ptr(const ga_desc* h, int n) { return h->tsem + (uint64_t)n * kSemStride; }
+static __device__ __forceinline__ uint64_t* page_bits(const ga_desc* h, uint64_t p) { return h->bits + p * kBinWords; }
 
 // ---------------------------------------------------------------------------
 // 2. bulk semaphore: word = (C:int32 << 32) | (D + 2^31), D = E - R (R-6)
@@ -133,14 +133,14 @@ static __device__ __forceinline__ void bsem_signal(uint64_t* s, uint32_t N, uint
     red_add_release(s, ((uint64_t)N << 32) - (uint64_t)B);
 }
 
-// try-wait (R-7): C -= N iff C >= N.
+// try-wait (R-7): C -= N iff C >= N.  One fetch-add: subtract,
+// and give the units back if the pre-image was short.
 static __device__ __forceinline__ bool bsem_trywait(uint64_t* s, uint32_t N) {
-    uint64_t w = ld_rlx(s);
-    while (sem_C(w) >= (int32_t)N) {
-        uint64_t old = a_cas(s, w, w - ((uint64_t)N << 32));
-        if (old == w) { fence(); return true; }
-        w = old;
-    }
+    if (sem_C(ld_rlx(s)) < (int32_t)N) return false;
+    const uint64_t dn = (uint64_t)N << 32;
+    uint64_t old = a_add(s, (uint64_t)0 - dn);
+    if (sem_C(old) >= (int32_t)N) { fence(); return true; }
+    a_add(s, dn);
     return false;
 }
 
@@ -151,26 +151,32 @@ static __device__ __forceinline__ bool bsem_trywait(uint64_t* s, uint32_t N) {
 // C < N and R <= C + E, i.e. C < N and C + D >= 0.
 template <class Spin>
 static __device__ __noinline__ int bsem_wait(uint64_t* s, uint32_t N, uint32_t B, Spin spin) {
-    uint64_t w = ld_rlx(s);
+    // Optimistic form of Alg. 1: one fetch-add C -= N decides on the pre-image.
+    //   pre C >= N           -> ACQUIRED (the common case: one atomic, no retry)
+    //   pre C + D < N        -> GROW: give C back, E += B - N
+    //   otherwise            -> reserve: give C back, R += N (C + D unchanged), spin
+    // The conversion adds keep C + D exact for reservations; an in-flight GROW
+    // conversion hides its B units for one round trip (others may over-produce,
+    // never over-grant).  DESIGN.md "Semaphore word" and tests/test_fa_model.py.
+    const uint64_t dn = (uint64_t)N << 32;
     for (;;) {
-        int32_t C = sem_C(w), D = sem_D(w);
-        uint64_t nw;
-        int res;
-        if ((int64_t)C + D < (int64_t)N) { nw = w + (uint64_t)(B - N); res = kGrow; }       // E += B - N
-        else if (C >= (int32_t)N) { nw = w - ((uint64_t)N << 32); res = kAcquired; }    // C -= N
-        else { nw = w - (uint64_t)N; res = kBlocked; }                                    // R += N
-        uint64_t old = a_cas(s, w, nw);
-        if (old != w) { w = old; continue; }
-        if (res != kBlocked) { fence(); return res; }
+        uint64_t old = a_add(s, (uint64_t)0 - dn);
+        int32_t C = sem_C(old), D = sem_D(old);
+        if (C >= (int32_t)N) { fence(); return kAcquired; }
+        if ((int64_t)C + D < (int64_t)N) {
+            a_add(s, dn + (uint64_t)(B - N));                                   // C += N, E += B - N
+            fence();
+            return kGrow;
+        }
+        uint64_t w = a_add(s, dn - (uint64_t)N) + dn - (uint64_t)N;            // C += N, R += N
         uint32_t ns = 64;
-        for (;;) {
-            w = ld_rlx(s);
-            if (!(sem_C(w) < (int32_t)N && (int64_t)sem_C(w) + sem_D(w) >= 0)) break;
+        while (sem_C(w) < (int32_t)N && (int64_t)sem_C(w) + sem_D(w) >= 0) {    // R-2
             spin();
             __nanosleep(ns);
             if (ns < 2048) ns <<= 1;
+            w = ld_rlx(s);
         }
-        w = a_add(s, (uint64_t)N) + (uint64_t)N;                                            // R -= N
+        a_add(s, (uint64_t)N);                                                  // R -= N
     }
 }
 struct NoSpin { __device__ void operator()() const {} };
@@ -259,19 +265,19 @@ static __device__ __noinline__ int64_t hb_find(const HB& b, uint32_t seed) {
     }
     return -1;
 }
-static __device__ __forceinline__ HB level_hb(const ga_dev_heap& h, int n) { HB b = hb_make(h.avail + h.lvl_off[n], h.lvl_words[n]); return b; }
-static __device__ __forceinline__ HB owned_hb(const ga_dev_heap& h, uint32_t A) {
-    uint32_t tw = hb_total_words(h.chunk_words);
-    return hb_make(h.owned + (uint64_t)A * tw, h.chunk_words);
+static __device__ __forceinline__ HB level_hb(const ga_desc* h, int n) { HB b = hb_make(h->avail + h->lvl_off[n], h->lvl_words[n]); return b; }
+static __device__ __forceinline__ HB owned_hb(const ga_desc* h, uint32_t A) {
+    uint32_t tw = hb_total_words(h->chunk_words);
+    return hb_make(h->owned + (uint64_t)A * tw, h->chunk_words);
 }
 
 // ---------------------------------------------------------------------------
 // 4. TBuddy
 // ---------------------------------------------------------------------------
-static __device__ __forceinline__ bool node_inside(const ga_dev_heap& h, int n, uint64_t i) { return ((i + 1) << n) <= h.pages; }
+static __device__ __forceinline__ bool node_inside(const ga_desc* h, int n, uint64_t i) { return ((i + 1) << n) <= h->pages; }
 
 // make node i of level n available (a split's right child, a freed root)
-static __device__ __forceinline__ void tree_publish(const ga_dev_heap& h, int n, uint64_t i, uint32_t expected) {
+static __device__ __forceinline__ void tree_publish(const ga_desc* h, int n, uint64_t i, uint32_t expected) {
     HB b = level_hb(h, n);
     hb_set(b, i);
     bsem_signal(tsem_ptr(h, n), 1, expected);            // C += 1 (and retire E if it was expected)
@@ -279,7 +285,7 @@ static __device__ __forceinline__ void tree_publish(const ga_dev_heap& h, int n,
 
 // claim up to `need` available nodes of level n (caller holds `need` units of
 // tsem[n]); claims from one word; returns the word index and the claimed mask
-static __device__ __noinline__ uint64_t tree_claim_word(const ga_dev_heap& h, int n, int need, uint32_t seed, uint64_t* word_out) {
+static __device__ __noinline__ uint64_t tree_claim_word(const ga_desc* h, int n, int need, uint32_t seed, uint64_t* word_out) {
     HB b = level_hb(h, n);
     uint32_t ns = 32;
     for (;;) {
@@ -304,10 +310,10 @@ static __device__ __noinline__ uint64_t tree_claim_word(const ga_dev_heap& h, in
 // Single-thread allocation of one order-o block, iterative:
 // climb while wait says GROW, claim at the first level that grants, split down.
 // Returns the node index at level o, or -1 (every E retracted).
-static __device__ __noinline__ int64_t tree_alloc_one(const ga_dev_heap& h, int o) {
+static __device__ __noinline__ int64_t tree_alloc_one(const ga_desc* h, int o) {
     int m = o;
     for (;;) {
-        if (m > (int)h.L) {                               // no parent: fail, retract E below
+        if (m > (int)h->L) {                               // no parent: fail, retract E below
             for (int k = o; k < m; k++) bsem_signal(tsem_ptr(h, k), 0, 1);
             return -1;
         }
@@ -328,13 +334,13 @@ static __device__ __noinline__ int64_t tree_alloc_one(const ga_dev_heap& h, int 
 // the buddy's available->busy transition both succeed, cascading (R-19);
 // otherwise mark it available with one CAS on the word that holds both
 // siblings (R-21), so two siblings never both end up available.
-static __device__ __noinline__ void tree_free(const ga_dev_heap& h, int n, uint64_t x) {
+static __device__ __noinline__ void tree_free(const ga_desc* h, int n, uint64_t x) {
     uint32_t ns = 32;
     for (;;) {
         HB b = level_hb(h, n);
         uint64_t* wp = &b.w[x >> 6];
         uint64_t xb = 1ull << (x & 63), yb = 1ull << ((x ^ 1) & 63);
-        bool root = (n >= (int)h.L) || !node_inside(h, n, x ^ 1);
+        bool root = (n >= (int)h->L) || !node_inside(h, n, x ^ 1);
         uint64_t w = ld_rlx(wp);
         if (!root && (w & yb)) {
             if (bsem_trywait(tsem_ptr(h, n), 1)) {
@@ -365,29 +371,29 @@ static __device__ __noinline__ void tree_free(const ga_dev_heap& h, int n, uint6
 static __device__ __forceinline__ uint32_t kind_bin(uint32_t A, int c) { return kKindBin | (A << 8) | (uint32_t)c; }
 
 // Reclamation (section 6) forward declarations
-static __device__ void reclaim_arena(const ga_dev_heap& h, uint32_t A, int budget);
+static __device__ void reclaim_arena(const ga_desc* h, uint32_t A, int budget);
 struct ArenaSpin {
-    const ga_dev_heap* h; uint32_t A;
-    __device__ void operator()() const { reclaim_arena(*h, A, 4); }
+    const ga_desc* h; uint32_t A;
+    __device__ void operator()() const { reclaim_arena(h, A, 4); }
 };
 
 // Take a new chunk from TBuddy for arena A, keep the first k pages, open the
 // rest.  Returns the chunk index or -1.
-static __device__ __noinline__ int64_t chunk_acquire(const ga_dev_heap& h, uint32_t A, uint32_t k) {
+static __device__ __noinline__ int64_t chunk_acquire(const ga_desc* h, uint32_t A, uint32_t k) {
     int64_t ch = tree_alloc_one(h, kChunkOrder);
     if (ch < 0) return -1;
-    st_rlx32(&h.chunk_owner[ch], A + 1);
+    st_rlx32(&h->chunk_owner[ch], A + 1);
     fence();
     hb_set(owned_hb(h, A), (uint64_t)ch);
     uint64_t keep = k >= 64 ? ~0ull : ((1ull << k) - 1);
-    a_and(&h.chunk_used[ch], keep);                       // open pages k..63
+    a_and(&h->chunk_used[ch], keep);                       // open pages k..63
     stat_add(h, kStatChunkGrow, 1);
     return ch;
 }
 
 // Claim up to `need` free pages of one chunk owned by A (caller holds `need`
 // units of psem[A]).  Returns the mask of pages claimed, chunk in *ch_out.
-static __device__ __noinline__ uint64_t page_claim(const ga_dev_heap& h, uint32_t A, int need, uint64_t* ch_out) {
+static __device__ __noinline__ uint64_t page_claim(const ga_desc* h, uint32_t A, int need, uint64_t* ch_out) {
     HB ob = owned_hb(h, A);
     uint32_t seed = scatter_seed();
     uint32_t ns = 32;
@@ -400,15 +406,15 @@ static __device__ __noinline__ uint64_t page_claim(const ga_dev_heap& h, uint32_
                 uint32_t bit = (uint32_t)(__ffsll((long long)ow) - 1);
                 ow &= ow - 1;
                 uint64_t ch = (uint64_t)j * 64 + bit;
-                uint64_t u = ld_rlx(&h.chunk_used[ch]);
+                uint64_t u = ld_rlx(&h->chunk_used[ch]);
                 while (~u) {
                     uint64_t m = lowest_bits(~u, need);
-                    uint64_t old = a_or(&h.chunk_used[ch], m);
+                    uint64_t old = a_or(&h->chunk_used[ch], m);
                     uint64_t got = m & ~old;
                     if (got) {
                         fence();
-                        if (ld_rlx32(&h.chunk_owner[ch]) != A + 1) {   // recycled chunk: undo
-                            a_and(&h.chunk_used[ch], ~got);
+                        if (ld_rlx32(&h->chunk_owner[ch]) != A + 1) {   // recycled chunk: undo
+                            a_and(&h->chunk_used[ch], ~got);
                             break;
                         }
                         *ch_out = ch;
@@ -424,29 +430,29 @@ static __device__ __noinline__ uint64_t page_claim(const ga_dev_heap& h, uint32_
 
 // Return page p (chunk ch, owner A) to its chunk: C += 1 on psem[A].  An empty
 // chunk goes back to TBuddy (R-23).
-static __device__ void chunk_release(const ga_dev_heap& h, uint64_t ch);
-static __device__ __noinline__ void page_release(const ga_dev_heap& h, uint64_t p) {
+static __device__ void chunk_release(const ga_desc* h, uint64_t ch);
+static __device__ __noinline__ void page_release(const ga_desc* h, uint64_t p) {
     uint64_t ch = p >> kChunkShift;
-    uint32_t A = ld_rlx32(&h.chunk_owner[ch]) - 1;
+    uint32_t A = ld_rlx32(&h->chunk_owner[ch]) - 1;
     uint64_t bit = 1ull << (p & (kChunkPages - 1));
-    uint64_t old = a_and(&h.chunk_used[ch], ~bit);
+    uint64_t old = a_and(&h->chunk_used[ch], ~bit);
     bsem_signal(psem_ptr(h, A), 1, 0);
     if ((old & ~bit) == 0) chunk_release(h, ch);
 }
 
 // An empty chunk back to the tree: try-wait all 64 page units, then take every
 // page with one CAS (0 -> all ones).  Failure leaves the chunk owned.
-static __device__ __noinline__ void chunk_release(const ga_dev_heap& h, uint64_t ch) {
-    uint32_t A = ld_rlx32(&h.chunk_owner[ch]) - 1;
-    if (A >= h.n_arenas) return;
+static __device__ __noinline__ void chunk_release(const ga_desc* h, uint64_t ch) {
+    uint32_t A = ld_rlx32(&h->chunk_owner[ch]) - 1;
+    if (A >= h->n_arenas) return;
     if (!bsem_trywait(psem_ptr(h, A), kChunkPages)) return;
-    if (a_cas(&h.chunk_used[ch], 0ull, ~0ull) != 0ull) { bsem_signal(psem_ptr(h, A), kChunkPages, 0); return; }
+    if (a_cas(&h->chunk_used[ch], 0ull, ~0ull) != 0ull) { bsem_signal(psem_ptr(h, A), kChunkPages, 0); return; }
     HB ob = owned_hb(h, A);
     uint64_t old = a_and(&ob.w[ch >> 6], ~(1ull << (ch & 63)));
     if ((old & ~(1ull << (ch & 63))) == 0) hb_word_zeroed(ob, (uint32_t)(ch >> 6));
-    a_exch(&h.chunk_cand[ch], 0);
-    for (int c = 0; c < kNcls; c++) a_exch(&h.chunk_nonfull[ch * kNcls + c], 0);
-    st_rlx32(&h.chunk_owner[ch], 0);
+    a_exch(&h->chunk_cand[ch], 0);
+    for (int c = 0; c < kNcls; c++) a_exch(&h->chunk_nonfull[ch * kNcls + c], 0);
+    st_rlx32(&h->chunk_owner[ch], 0);
     fence();
     stat_add(h, kStatChunkReclaim, 1);
     tree_free(h, kChunkOrder, ch);
@@ -454,8 +460,8 @@ static __device__ __noinline__ void chunk_release(const ga_dev_heap& h, uint64_t
 
 // Make page p a bin of class c for arena A.  The group keeps slots [0, take);
 // the others are opened (bitmap was all ones).  Returns true if slots remain.
-static __device__ __forceinline__ bool bin_init(const ga_dev_heap& h, uint64_t p, uint32_t A, int c, uint32_t take) {
-    st_rlx32(&h.kind[p], kind_bin(A, c));
+static __device__ __forceinline__ bool bin_init(const ga_desc* h, uint64_t p, uint32_t A, int c, uint32_t take) {
+    st_rlx32(&h->kind[p], kind_bin(A, c));
     fence();
     uint64_t* bw = page_bits(h, p);
     for (int w = 0; w < words_of(c); w++) {
@@ -468,8 +474,8 @@ static __device__ __forceinline__ bool bin_init(const ga_dev_heap& h, uint64_t p
     return take < slots_of(c);
 }
 
-static __device__ __forceinline__ void nonfull_set(const ga_dev_heap& h, uint64_t p, int c) {
-    uint64_t* nf = &h.chunk_nonfull[(p >> kChunkShift) * kNcls + c];
+static __device__ __forceinline__ void nonfull_set(const ga_desc* h, uint64_t p, int c) {
+    uint64_t* nf = &h->chunk_nonfull[(p >> kChunkShift) * kNcls + c];
     uint64_t bit = 1ull << (p & (kChunkPages - 1));
     if (!(ld_rlx(nf) & bit)) a_or(nf, bit);
 }
@@ -478,20 +484,20 @@ static __device__ __forceinline__ bool page_full(const uint64_t w[4], int c) {
     return true;
 }
 // clear-then-recheck: drop p from the nonfull set only if it is really full
-static __device__ __noinline__ void nonfull_clear_if_full(const ga_dev_heap& h, uint64_t p, int c, uint32_t A) {
-    uint64_t* nf = &h.chunk_nonfull[(p >> kChunkShift) * kNcls + c];
+static __device__ __noinline__ void nonfull_clear_if_full(const ga_desc* h, uint64_t p, int c, uint32_t A) {
+    uint64_t* nf = &h->chunk_nonfull[(p >> kChunkShift) * kNcls + c];
     uint64_t bit = 1ull << (p & (kChunkPages - 1));
     a_and(nf, ~bit);
     fence();
     uint64_t w[4];
     ld_bitmap(page_bits(h, p), w);
-    if (ld_rlx32(&h.kind[p]) == kind_bin(A, c) && !page_full(w, c)) a_or(nf, bit);
+    if (ld_rlx32(&h->kind[p]) == kind_bin(A, c) && !page_full(w, c)) a_or(nf, bit);
 }
 
 // Try to claim up to `need` slots of page p (must be an (A, c) bin) from one
 // word.  Returns the claimed mask and word index; 0 if the page had none.
-static __device__ __noinline__ uint64_t bin_claim_page(const ga_dev_heap& h, uint64_t p, uint32_t A, int c, int need, int* word_out) {
-    if (ld_rlx32(&h.kind[p]) != kind_bin(A, c)) return 0;
+static __device__ __noinline__ uint64_t bin_claim_page(const ga_desc* h, uint64_t p, uint32_t A, int c, int need, int* word_out) {
+    if (ld_rlx32(&h->kind[p]) != kind_bin(A, c)) return 0;
     uint64_t* bw = page_bits(h, p);
     uint64_t w[4];
     ld_bitmap(bw, w);
@@ -503,7 +509,7 @@ static __device__ __noinline__ uint64_t bin_claim_page(const ga_dev_heap& h, uin
             uint64_t got = m & ~old;
             if (got) {
                 fence();
-                if (ld_rlx32(&h.kind[p]) != kind_bin(A, c)) {     // recycled page: undo as a free
+                if (ld_rlx32(&h->kind[p]) != kind_bin(A, c)) {     // recycled page: undo as a free
                     a_and(&bw[i], ~got);
                     return 0;
                 }
@@ -523,7 +529,7 @@ static __device__ __noinline__ uint64_t bin_claim_page(const ga_dev_heap& h, uin
 
 // Find a bin of (A, c) with a free slot: the arena hint first, then every
 // owned chunk's nonfull mask.  Returns the page or kNull.
-static __device__ __noinline__ uint64_t bin_find(const ga_dev_heap& h, uint32_t A, int c, uint32_t seed) {
+static __device__ __noinline__ uint64_t bin_find(const ga_desc* h, uint32_t A, int c, uint32_t seed) {
     HB ob = owned_hb(h, A);
     for (uint32_t t = 0; t < ob.n[0]; t++) {
         uint32_t j = (seed + t) % ob.n[0];
@@ -532,14 +538,14 @@ static __device__ __noinline__ uint64_t bin_find(const ga_dev_heap& h, uint32_t 
             uint32_t bit = (uint32_t)(__ffsll((long long)ow) - 1);
             ow &= ow - 1;
             uint64_t ch = (uint64_t)j * 64 + bit;
-            uint64_t nf = ld_rlx(&h.chunk_nonfull[ch * kNcls + c]);
+            uint64_t nf = ld_rlx(&h->chunk_nonfull[ch * kNcls + c]);
             while (nf) {
                 uint32_t pb = (uint32_t)(__ffsll((long long)nf) - 1);
                 nf &= nf - 1;
                 uint64_t p = ch * kChunkPages + pb;
                 uint64_t w[4];
                 ld_bitmap(page_bits(h, p), w);
-                if (ld_rlx32(&h.kind[p]) == kind_bin(A, c) && !page_full(w, c)) return p;
+                if (ld_rlx32(&h->kind[p]) == kind_bin(A, c) && !page_full(w, c)) return p;
                 nonfull_clear_if_full(h, p, c, A);        // stale bit
             }
         }
@@ -553,8 +559,8 @@ static __device__ __noinline__ uint64_t bin_find(const ga_dev_heap& h, uint32_t 
 // ---------------------------------------------------------------------------
 // Reclaim page p if it is an empty bin: try-wait all its slots (R-22), then
 // take every slot word with a CAS (all free -> all ones).
-static __device__ __noinline__ bool bin_reclaim(const ga_dev_heap& h, uint64_t p) {
-    uint32_t k = ld_rlx32(&h.kind[p]);
+static __device__ __noinline__ bool bin_reclaim(const ga_desc* h, uint64_t p) {
+    uint32_t k = ld_rlx32(&h->kind[p]);
     if ((k & 0xC0000000u) != kKindBin) return false;
     uint32_t A = (k >> 8) & 0xFFFFu;
     int c = (int)(k & 0xFF);
@@ -574,25 +580,25 @@ static __device__ __noinline__ bool bin_reclaim(const ga_dev_heap& h, uint64_t p
         bsem_signal(sem_ptr(h, A, c), slots, 0);
         return false;
     }
-    a_and(&h.chunk_nonfull[(p >> kChunkShift) * kNcls + c], ~(1ull << (p & (kChunkPages - 1))));
-    st_rlx32(&h.kind[p], 0);
+    a_and(&h->chunk_nonfull[(p >> kChunkShift) * kNcls + c], ~(1ull << (p & (kChunkPages - 1))));
+    st_rlx32(&h->kind[p], 0);
     fence();
     stat_add(h, kStatBinReclaim, 1);
     page_release(h, p);
     return true;
 }
 
-static __device__ __forceinline__ void mark_candidate(const ga_dev_heap& h, uint64_t p, uint32_t A) {
-    uint64_t* cw = &h.chunk_cand[p >> kChunkShift];
+static __device__ __forceinline__ void mark_candidate(const ga_desc* h, uint64_t p, uint32_t A) {
+    uint64_t* cw = &h->chunk_cand[p >> kChunkShift];
     uint64_t bit = 1ull << (p & (kChunkPages - 1));
     if (!(ld_rlx(cw) & bit)) a_or(cw, bit);
     fence();
-    if (!ld_rlx(&h.cand_any[A * kSemStride])) a_or(&h.cand_any[A * kSemStride], 1);
+    if (!ld_rlx(&h->cand_any[A * kSemStride])) a_or(&h->cand_any[A * kSemStride], 1);
 }
 
 // Reclaim up to `budget` candidate bins of arena A (budget < 0: all).
-static __device__ __noinline__ void reclaim_arena(const ga_dev_heap& h, uint32_t A, int budget) {
-    uint64_t* any = &h.cand_any[A * kSemStride];
+static __device__ __noinline__ void reclaim_arena(const ga_desc* h, uint32_t A, int budget) {
+    uint64_t* any = &h->cand_any[A * kSemStride];
     if (!ld_rlx(any)) return;
     a_exch(any, 0);
     fence();
@@ -604,13 +610,13 @@ static __device__ __noinline__ void reclaim_arena(const ga_dev_heap& h, uint32_t
             uint32_t bit = (uint32_t)(__ffsll((long long)ow) - 1);
             ow &= ow - 1;
             uint64_t ch = (uint64_t)j * 64 + bit;
-            if (!ld_rlx(&h.chunk_cand[ch])) continue;
+            if (!ld_rlx(&h->chunk_cand[ch])) continue;
             if (budget == 0) { left = true; break; }
-            uint64_t cm = a_exch(&h.chunk_cand[ch], 0);
+            uint64_t cm = a_exch(&h->chunk_cand[ch], 0);
             while (cm) {
                 uint32_t pb = (uint32_t)(__ffsll((long long)cm) - 1);
                 cm &= cm - 1;
-                if (budget == 0) { a_or(&h.chunk_cand[ch], 1ull << pb); left = true; continue; }
+                if (budget == 0) { a_or(&h->chunk_cand[ch], 1ull << pb); left = true; continue; }
                 bin_reclaim(h, ch * kChunkPages + pb);
                 if (budget > 0) budget--;
             }
@@ -619,21 +625,21 @@ static __device__ __noinline__ void reclaim_arena(const ga_dev_heap& h, uint32_t
     }
     if (left) { fence(); a_or(any, 1); }
 }
-static __device__ __noinline__ void reclaim_all(const ga_dev_heap& h) {
-    for (uint32_t A = 0; A < h.n_arenas; A++) reclaim_arena(h, A, -1);
+static __device__ __noinline__ void reclaim_all(const ga_desc* h) {
+    for (uint32_t A = 0; A < h->n_arenas; A++) reclaim_arena(h, A, -1);
 }
 
 // ---------------------------------------------------------------------------
 // 7. front end
 // ---------------------------------------------------------------------------
 // size -> key: 0..7 bin class, 8 + order for TBuddy, -1 for NULL
-static __device__ __forceinline__ int size_key(const ga_dev_heap& h, uint64_t n) {
-    if (n == 0 || n > (h.pages << kPageShift)) return -1;                  // R-15
+static __device__ __forceinline__ int size_key(const ga_desc* h, uint64_t n) {
+    if (n == 0 || n > (h->pages << kPageShift)) return -1;                  // R-15
     if (n <= 16) return 0;
     int lg = 64 - __clzll((long long)(n - 1));                            // ceil(log2 n), R-14
     if (lg <= 11) return lg - kMinShift;                                  // <= 2048 B: bins (R-12)
     int o = lg - kPageShift;
-    if (o > (int)h.L) return -1;
+    if (o > (int)h->L) return -1;
     return kNcls + o;
 }
 
@@ -669,17 +675,17 @@ struct BinLeader {
     uint32_t seed;
 };
 
-static __device__ __noinline__ Grant bin_leader_step(const ga_dev_heap& h, BinLeader& L) {
+static __device__ __noinline__ Grant bin_leader_step(const ga_desc* h, BinLeader& L) {
     Grant g; g.kind = 3; g.base = L.served; g.count = 0; g.unit = 0; g.mask = 0; g.word = 0;
     uint32_t slots = slots_of(L.c);
     if (L.phase == 0) {
         L.Bp = slots * ((L.N + slots - 1) / slots);                          // R-8
-        int r = bsem_wait(sem_ptr(h, L.A, L.c), L.N, L.Bp, ArenaSpin{&h, L.A});
-        if (r == kAcquired) { L.phase = 1; L.hint = ld_rlx32(&h.hint[L.A * kNcls + L.c]); }
+        int r = bsem_wait(sem_ptr(h, L.A, L.c), L.N, L.Bp, ArenaSpin{h, L.A});
+        if (r == kAcquired) { L.phase = 1; L.hint = ld_rlx32(&h->hint[L.A * kNcls + L.c]); }
         else {
             // GROW: B'/slots new bins; pages accounted on the arena's page semaphore
             uint32_t k = L.Bp / slots;
-            int rp = bsem_wait(psem_ptr(h, L.A), k, kChunkPages, ArenaSpin{&h, L.A});
+            int rp = bsem_wait(psem_ptr(h, L.A), k, kChunkPages, ArenaSpin{h, L.A});
             if (rp == kGrow) {
                 reclaim_arena(h, L.A, -1);                 // delegated work before a new chunk
                 int64_t ch = chunk_acquire(h, L.A, k);
@@ -704,7 +710,7 @@ static __device__ __noinline__ Grant bin_leader_step(const ga_dev_heap& h, BinLe
                 g.kind = 1; g.unit = (uint64_t)ch; g.mask = pm; g.count = L.N; g.word = (int)slots;
                 L.served = L.N;
                 L.hint = (uint64_t)ch * kChunkPages + k - 1;
-                st_rlx32(&h.hint[L.A * kNcls + L.c], (uint32_t)L.hint);
+                st_rlx32(&h->hint[L.A * kNcls + L.c], (uint32_t)L.hint);
                 bsem_signal(sem_ptr(h, L.A, L.c), L.Bp - L.N, L.Bp - L.N);
                 L.phase = 3;
                 return g;
@@ -732,7 +738,7 @@ static __device__ __noinline__ Grant bin_leader_step(const ga_dev_heap& h, BinLe
         g.kind = 1; g.unit = ch; g.mask = pm; g.count = serve; g.word = (int)slots;
         L.served += serve;
         if (L.pages_left == 0) {
-            st_rlx32(&h.hint[L.A * kNcls + L.c], (uint32_t)L.hint);
+            st_rlx32(&h->hint[L.A * kNcls + L.c], (uint32_t)L.hint);
             bsem_signal(sem_ptr(h, L.A, L.c), L.Bp - L.N, L.Bp - L.N);
             L.phase = 3;
         }
@@ -742,7 +748,7 @@ static __device__ __noinline__ Grant bin_leader_step(const ga_dev_heap& h, BinLe
         uint32_t ns = 32;
         for (;;) {
             uint64_t p = L.hint;
-            if (p < h.pages) {
+            if (p < h->pages) {
                 int wi;
                 uint64_t got = bin_claim_page(h, p, L.A, L.c, (int)(L.N - L.served), &wi);
                 if (got) {
@@ -751,7 +757,7 @@ static __device__ __noinline__ Grant bin_leader_step(const ga_dev_heap& h, BinLe
                     L.served += n;
                     if (L.served == L.N) {
                         L.phase = 3;
-                        if (ld_rlx32(&h.hint[L.A * kNcls + L.c]) != (uint32_t)p) st_rlx32(&h.hint[L.A * kNcls + L.c], (uint32_t)p);
+                        if (ld_rlx32(&h->hint[L.A * kNcls + L.c]) != (uint32_t)p) st_rlx32(&h->hint[L.A * kNcls + L.c], (uint32_t)p);
                     }
                     return g;
                 }
@@ -769,17 +775,17 @@ static __device__ __noinline__ Grant bin_leader_step(const ga_dev_heap& h, BinLe
 
 // Per-lane slow path (R-26, R-27): N = 1 waits; after local growth fails,
 // drain reclamation, then take pages and slots from other arenas before NULL.
-static __device__ __noinline__ uint64_t bin_malloc_lane(const ga_dev_heap& h, uint32_t A0, int c) {
+static __device__ __noinline__ uint64_t bin_malloc_lane(const ga_desc* h, uint32_t A0, int c) {
     uint32_t slots = slots_of(c);
     uint64_t csz = 16ull << c;
     for (int attempt = 0; attempt < 2; attempt++) {
-        int r = bsem_wait(sem_ptr(h, A0, c), 1, slots, ArenaSpin{&h, A0});
+        int r = bsem_wait(sem_ptr(h, A0, c), 1, slots, ArenaSpin{h, A0});
         if (r == kAcquired) {
             uint32_t seed = scatter_seed();
             uint32_t ns = 32;
-            uint64_t p = ld_rlx32(&h.hint[A0 * kNcls + c]);
+            uint64_t p = ld_rlx32(&h->hint[A0 * kNcls + c]);
             for (;;) {
-                if (p < h.pages) {
+                if (p < h->pages) {
                     int wi;
                     uint64_t got = bin_claim_page(h, p, A0, c, 1, &wi);
                     if (got) return (p << kPageShift) + (uint64_t)(wi * 64 + __ffsll((long long)got) - 1) * csz;
@@ -788,7 +794,7 @@ static __device__ __noinline__ uint64_t bin_malloc_lane(const ga_dev_heap& h, ui
                 if (p == kNull) { __nanosleep(ns); if (ns < 1024) ns <<= 1; seed = hash32(seed + 3); }
             }
         }
-        int rp = bsem_wait(psem_ptr(h, A0), 1, kChunkPages, ArenaSpin{&h, A0});
+        int rp = bsem_wait(psem_ptr(h, A0), 1, kChunkPages, ArenaSpin{h, A0});
         uint64_t p = kNull;
         if (rp == kAcquired) {
             uint64_t ch;
@@ -803,7 +809,7 @@ static __device__ __noinline__ uint64_t bin_malloc_lane(const ga_dev_heap& h, ui
         if (p != kNull) {
             if (bin_init(h, p, A0, c, 1)) nonfull_set(h, p, c);
             stat_add(h, kStatBinGrow, 1);
-            st_rlx32(&h.hint[A0 * kNcls + c], (uint32_t)p);
+            st_rlx32(&h->hint[A0 * kNcls + c], (uint32_t)p);
             bsem_signal(sem_ptr(h, A0, c), slots - 1, slots - 1);
             return p << kPageShift;
         }
@@ -813,8 +819,8 @@ static __device__ __noinline__ uint64_t bin_malloc_lane(const ga_dev_heap& h, ui
     // every page source first (they only shrink in malloc-only phases), then
     // every arena's bins of this class: a malloc fails only if no arena can
     // serve it (R-26)
-    for (uint32_t t = 1; t <= h.n_arenas; t++) {
-        uint32_t B = (A0 + t) % h.n_arenas;
+    for (uint32_t t = 1; t <= h->n_arenas; t++) {
+        uint32_t B = (A0 + t) % h->n_arenas;
         if (bsem_wait(psem_ptr(h, B), 1, 1, NoSpin()) == kAcquired) {
             uint64_t ch;
             uint64_t pm = page_claim(h, B, 1, &ch);
@@ -825,14 +831,14 @@ static __device__ __noinline__ uint64_t bin_malloc_lane(const ga_dev_heap& h, ui
             return p << kPageShift;
         }
     }
-    for (uint32_t t = 1; t <= h.n_arenas; t++) {
-        uint32_t B = (A0 + t) % h.n_arenas;
+    for (uint32_t t = 1; t <= h->n_arenas; t++) {
+        uint32_t B = (A0 + t) % h->n_arenas;
         if (bsem_wait(sem_ptr(h, B, c), 1, 1, NoSpin()) == kAcquired) {
             uint32_t seed = scatter_seed();
             uint32_t ns = 32;
-            uint64_t p = ld_rlx32(&h.hint[B * kNcls + c]);
+            uint64_t p = ld_rlx32(&h->hint[B * kNcls + c]);
             for (;;) {
-                if (p < h.pages) {
+                if (p < h->pages) {
                     int wi;
                     uint64_t got = bin_claim_page(h, p, B, c, 1, &wi);
                     if (got) return (p << kPageShift) + (uint64_t)(wi * 64 + __ffsll((long long)got) - 1) * csz;
@@ -852,13 +858,13 @@ struct TreeLeader {
 };
 static __device__ __forceinline__ uint32_t ceil_half(uint32_t x) { return (x + 1) >> 1; }
 
-static __device__ __noinline__ Grant tree_leader_step(const ga_dev_heap& h, TreeLeader& L) {
+static __device__ __noinline__ Grant tree_leader_step(const ga_desc* h, TreeLeader& L) {
     Grant g; g.kind = 3; g.base = L.served; g.count = 0; g.unit = 0; g.mask = 0; g.word = 0;
     if (L.phase == 0) {
         uint32_t Nk = L.N;
         int m = L.o;
         for (;;) {
-            if (m > (int)h.L) {                              // nothing to grow from: retract E
+            if (m > (int)h->L) {                              // nothing to grow from: retract E
                 uint32_t nk = L.N;
                 for (int k = L.o; k < m; k++) { bsem_signal(tsem_ptr(h, k), 0, 2 * ceil_half(nk) - nk); nk = ceil_half(nk); }
                 g.kind = 4;
@@ -902,7 +908,7 @@ static __device__ __noinline__ Grant tree_leader_step(const ga_dev_heap& h, Tree
 
 // ---- the group driver --------------------------------------------------------
 // Every lane of `grp` calls this with the same key; returns this lane's offset.
-static __device__ __forceinline__ uint64_t group_malloc(const ga_dev_heap& h, unsigned grp, int key) {
+static __device__ __forceinline__ uint64_t group_malloc(const ga_desc* h, unsigned grp, int key) {
     const int lane = (int)lane_id();
     const int leader = __ffs(grp) - 1;
     const uint32_t N = __popc(grp);
@@ -933,7 +939,7 @@ static __device__ __forceinline__ uint64_t group_malloc(const ga_dev_heap& h, un
                         }
                         if (x >= 0) {
                             uint64_t pg = (uint64_t)x << o;
-                            st_rlx32(&h.kind[pg], kKindTree | (uint32_t)o);
+                            st_rlx32(&h->kind[pg], kKindTree | (uint32_t)o);
                             my = pg << kPageShift;
                         } else stat_add(h, kStatFail, 1);
                     }
@@ -955,7 +961,7 @@ static __device__ __forceinline__ uint64_t group_malloc(const ga_dev_heap& h, un
                 uint64_t x = g.unit * 64 + nth_set(g.mask, r >> s);
                 uint64_t node = (x << s) + (r & ((1u << s) - 1));
                 uint64_t pg = node << o;
-                st_rlx32(&h.kind[pg], kKindTree | (uint32_t)o);
+                st_rlx32(&h->kind[pg], kKindTree | (uint32_t)o);
                 my = pg << kPageShift;
             }
         }
@@ -963,7 +969,7 @@ static __device__ __forceinline__ uint64_t group_malloc(const ga_dev_heap& h, un
     return my;
 }
 
-static __device__ __noinline__ uint64_t ga_malloc_off(const ga_dev_heap& h, uint64_t n) {
+static __device__ __noinline__ uint64_t ga_malloc_off(const ga_desc* h, uint64_t n) {
     unsigned act = __activemask();
     int key = size_key(h, n);
     unsigned grp = __match_any_sync(act, key);
@@ -973,17 +979,17 @@ static __device__ __noinline__ uint64_t ga_malloc_off(const ga_dev_heap& h, uint
 
 // free: TBuddy blocks per lane; bin slots grouped per bitmap word (one
 // atomicAnd) and per (arena, class) (one signal)
-static __device__ __noinline__ void ga_free_off(const ga_dev_heap& h, uint64_t off) {
+static __device__ __noinline__ void ga_free_off(const ga_desc* h, uint64_t off) {
     unsigned act = __activemask();
     uint32_t k = 0;
     uint64_t p = 0;
-    if (off != kNull) { p = off >> kPageShift; k = ld_rlx32(&h.kind[p]); }
+    if (off != kNull) { p = off >> kPageShift; k = ld_rlx32(&h->kind[p]); }
     bool is_bin = (off != kNull) && ((k & 0xC0000000u) == kKindBin);
     unsigned bins = __ballot_sync(act, is_bin);
     if (off != kNull && !is_bin) {
         // TBuddy block (page aligned); order from the page kind (R-18)
         int o = (int)(k & 0xFF);
-        st_rlx32(&h.kind[p], 0);
+        st_rlx32(&h->kind[p], 0);
         fence();
         tree_free(h, o, p >> o);
     }

@@ -38,28 +38,28 @@ __global__ void k_fill_u32(uint32_t* p, uint64_t n, uint32_t v) {
     for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) p[i] = v;
 }
 // quiesce step 1: every empty bin back to its chunk (and empty chunks to the tree)
-__global__ void k_quiesce_bins(ga_dev_heap h) {
-    for (uint64_t p = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; p < h.pages; p += (uint64_t)gridDim.x * blockDim.x) {
-        uint32_t k = h.kind[p];
+__global__ void k_quiesce_bins(const ga_desc* h) {
+    for (uint64_t p = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; p < h->pages; p += (uint64_t)gridDim.x * blockDim.x) {
+        uint32_t k = h->kind[p];
         if ((k & 0xC0000000u) == kKindBin) bin_reclaim(h, p);
     }
 }
 // quiesce step 2: chunks whose pages are all free go back to TBuddy
-__global__ void k_quiesce_chunks(ga_dev_heap h) {
-    for (uint64_t ch = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; ch < h.nchunks; ch += (uint64_t)gridDim.x * blockDim.x) {
-        if (h.chunk_owner[ch] != 0 && ld_rlx(&h.chunk_used[ch]) == 0) chunk_release(h, ch);
+__global__ void k_quiesce_chunks(const ga_desc* h) {
+    for (uint64_t ch = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; ch < h->nchunks; ch += (uint64_t)gridDim.x * blockDim.x) {
+        if (h->chunk_owner[ch] != 0 && ld_rlx(&h->chunk_used[ch]) == 0) chunk_release(h, ch);
     }
 }
-__global__ void k_quiesce_clear(ga_dev_heap h) {
+__global__ void k_quiesce_clear(const ga_desc* h) {
     uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-    if (i < h.nchunks) h.chunk_cand[i] = 0;
-    if (i < h.n_arenas) h.cand_any[i * kSemStride] = 0;
+    if (i < h->nchunks) h->chunk_cand[i] = 0;
+    if (i < h->n_arenas) h->cand_any[i * kSemStride] = 0;
 }
 
 inline int grid_for(uint64_t n) { uint64_t b = (n + 255) / 256; return (int)(b > 4096 ? 4096 : (b ? b : 1)); }
 
 ga_status init_heap(ga_heap_t h, cudaStream_t s) {
-    ga_dev_heap& d = h->dev;
+    ga_desc& d = h->dev;
     auto chk = [](cudaError_t e) { return e == cudaSuccess; };
     k_fill_u64<<<grid_for(d.pages * kBinWords), 256, 0, s>>>(d.bits, d.pages * kBinWords, ~0ull);
     k_fill_u32<<<grid_for(d.pages), 256, 0, s>>>(d.kind, d.pages, 0u);
@@ -74,6 +74,7 @@ ga_status init_heap(ga_heap_t h, cudaStream_t s) {
     k_fill_u64<<<grid_for((uint64_t)d.n_arenas * kSemStride), 256, 0, s>>>(d.cand_any, (uint64_t)d.n_arenas * kSemStride, 0ull);
     k_fill_u64<<<1, 32, 0, s>>>(d.stats, 16, 0ull);
     if (!chk(cudaGetLastError())) return GA_ECUDA;
+    if (!chk(cudaMemcpyAsync(h->ddesc, &h->dev, sizeof(ga_desc), cudaMemcpyHostToDevice, s))) return GA_ECUDA;
     if (!chk(cudaMemcpyAsync(d.avail, h->avail_init.data(), h->avail_words * 8, cudaMemcpyHostToDevice, s))) return GA_ECUDA;
     if (!chk(cudaMemcpyAsync(d.tsem, h->tsem_init.data(), h->tsem_init.size() * 8, cudaMemcpyHostToDevice, s))) return GA_ECUDA;
     h->peak_reserved_pages = 0;
@@ -129,7 +130,7 @@ ga_status ga_heap_create(int device, ga_stream_t stream, void* buf, size_t bytes
     ga_heap_t h = new (std::nothrow) ga_heap_s();
     if (!h) return GA_ENOMEM;
     h->device = device;
-    ga_dev_heap& d = h->dev;
+    ga_desc& d = h->dev;
     d.pages = nchunks * kChunkPages;
     d.nchunks = nchunks;
     uint32_t L = 0;
@@ -151,6 +152,7 @@ ga_status ga_heap_create(int device, ga_stream_t stream, void* buf, size_t bytes
     h->avail_words = aw;
     h->owned_words = (uint64_t)d.n_arenas * hb_total_words(d.chunk_words);
     Carve cv;
+    uint64_t o_desc = cv.take<ga_desc>(1);
     uint64_t o_bits = cv.take<uint64_t>(d.pages * kBinWords);
     uint64_t o_kind = cv.take<uint32_t>(d.pages);
     uint64_t o_used = cv.take<uint64_t>(nchunks);
@@ -175,6 +177,7 @@ ga_status ga_heap_create(int device, ga_stream_t stream, void* buf, size_t bytes
         d.base = (char*)up((uint64_t)(uintptr_t)h->pool_raw, kBaseAlign);
     }
     char* m = h->meta;
+    h->ddesc = (ga_desc*)(m + o_desc);
     d.bits = (uint64_t*)(m + o_bits);
     d.kind = (uint32_t*)(m + o_kind);
     d.chunk_used = (uint64_t*)(m + o_used);
@@ -230,7 +233,8 @@ ga_status ga_heap_reset(ga_heap_t h, ga_stream_t stream) {
 
 ga_status ga_heap_device(ga_heap_t h, ga_dev_heap* out) {
     if (!h || !out) return GA_EINVAL;
-    *out = h->dev;
+    out->desc = h->ddesc;
+    out->base = h->dev.base;
     return GA_OK;
 }
 
@@ -245,16 +249,16 @@ ga_status ga_heap_info(ga_heap_t h, uint64_t* heap_bytes, void** base, uint64_t*
 ga_status ga_heap_quiesce(ga_heap_t h, ga_stream_t stream) {
     if (!h) return GA_EINVAL;
     cudaStream_t s = (cudaStream_t)stream;
-    k_quiesce_bins<<<grid_for(h->dev.pages), 256, 0, s>>>(h->dev);
-    k_quiesce_chunks<<<grid_for(h->dev.nchunks), 256, 0, s>>>(h->dev);
+    k_quiesce_bins<<<grid_for(h->dev.pages), 256, 0, s>>>(h->ddesc);
+    k_quiesce_chunks<<<grid_for(h->dev.nchunks), 256, 0, s>>>(h->ddesc);
     uint64_t n = h->dev.nchunks > h->dev.n_arenas ? h->dev.nchunks : h->dev.n_arenas;
-    k_quiesce_clear<<<(int)((n + 255) / 256), 256, 0, s>>>(h->dev);
+    k_quiesce_clear<<<(int)((n + 255) / 256), 256, 0, s>>>(h->ddesc);
     return cudaGetLastError() == cudaSuccess ? GA_OK : GA_ECUDA;
 }
 
 ga_status ga_reserved_pages(ga_heap_t h, ga_stream_t stream, uint64_t* out) {
     if (!h || !out) return GA_EINVAL;
-    const ga_dev_heap& d = h->dev;
+    const ga_desc& d = h->dev;
     std::vector<uint64_t> av(h->avail_words);
     if (cudaMemcpyAsync(av.data(), d.avail, h->avail_words * 8, cudaMemcpyDeviceToHost, (cudaStream_t)stream) != cudaSuccess) return GA_ECUDA;
     if (cudaStreamSynchronize((cudaStream_t)stream) != cudaSuccess) return GA_ECUDA;
@@ -298,7 +302,7 @@ ga_status ga_stats(ga_heap_t h, ga_stream_t stream, ga_stats_t* out) {
 
 ga_status ga_heap_snapshot(ga_heap_t h, ga_stream_t stream, void* host, size_t cap, size_t* used) {
     if (!h || !used) return GA_EINVAL;
-    const ga_dev_heap& d = h->dev;
+    const ga_desc& d = h->dev;
     cudaStream_t s = (cudaStream_t)stream;
     std::vector<uint64_t> bits(d.pages * kBinWords), used_(d.nchunks), nonfull(1), cand(d.nchunks);
     std::vector<uint32_t> kind(d.pages), owner(d.nchunks);

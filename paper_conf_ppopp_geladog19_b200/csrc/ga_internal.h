@@ -11,7 +11,8 @@ struct ga_heap_s {
     char* pool_raw = nullptr;      // owned pool allocation (nullptr if borrowed)
     char* meta = nullptr;          // metadata allocation (R-29)
     size_t meta_bytes = 0;
-    ga_dev_heap dev{};
+    ga_desc dev{};                 // host copy of the descriptor
+    ga_desc* ddesc = nullptr;      // device copy (start of the metadata allocation)
     std::vector<uint64_t> avail_init;   // host image of the tree bitmaps (empty heap)
     std::vector<uint64_t> tsem_init;
     uint64_t avail_words = 0;

@@ -1,0 +1,37 @@
+"""Run the timed trace kernel a few times (for ncu captures).  Not a bench number."""
+import argparse
+import os
+import sys
+
+import numpy as np
+import torch
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import tracegen  # noqa: E402
+from paper_conf_ppopp_geladog19_b200.runner import GpuHeap, run_timed  # noqa: E402
+
+ap = argparse.ArgumentParser()
+ap.add_argument("--workload", default="d4")
+ap.add_argument("--size", type=int, default=16)
+ap.add_argument("--rounds", type=int, default=16)
+ap.add_argument("--reps", type=int, default=3)
+ap.add_argument("--cuda", action="store_true")
+a = ap.parse_args()
+if a.workload == "d4":
+    t = tracegen.d4_mixed("pressure", R=a.rounds)
+else:
+    t = tracegen.d3_uniform(a.size, R=a.rounds)
+torch.cuda.set_device(0)
+heap = None if a.cuda else GpuHeap(t.heap_bytes)
+if a.cuda:
+    import paper_conf_ppopp_geladog19_b200 as ga
+    ga.ga_cuda_set_heap_limit(t.heap_bytes)
+d = torch.from_numpy(t.sizes.view(np.int32)).cuda()
+c = torch.zeros(8, dtype=torch.int64, device="cuda")
+for i in range(a.reps):
+    s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    s.record()
+    run_timed(heap, d, t.R, t.T, t.D, c)
+    e.record()
+    e.synchronize()
+    print(f"rep {i}: {s.elapsed_time(e):.2f} ms, counts {c.cpu().numpy()[:4]}", flush=True)
