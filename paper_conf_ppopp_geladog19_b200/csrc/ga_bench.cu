@@ -8,6 +8,7 @@
 
 #include <cstdint>
 #include <cstdio>
+#include <cstdlib>
 
 #include "ga.h"
 #include "ga_bench.h"
@@ -135,8 +136,8 @@ __global__ void __launch_bounds__(256) k_phase(P al, const uint32_t* sizes, uint
 }
 
 // timing mode: every round in one kernel
-template <class P>
-__global__ void __launch_bounds__(256) k_timed(P al, const uint32_t* __restrict__ sizes, uint32_t R, uint32_t T, uint32_t D,
+template <class P, int MINB>
+__global__ void __launch_bounds__(256, MINB) k_timed(P al, const uint32_t* __restrict__ sizes, uint32_t R, uint32_t T, uint32_t D,
                                                uint64_t* counts) {
     uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
     if (t >= T) return;
@@ -293,6 +294,12 @@ __global__ void k_bsem_init(uint32_t n_sems, uint64_t* sems, uint32_t variant) {
     if (i < n_sems * 4 + 4) sems[i] = (variant <= 1 && i < n_sems * 4) ? 0x80000000ull : 0ull;
 }
 
+// resident 256-thread blocks per SM the timed kernel is compiled for (register
+// budget 65536 / (256 * minB)); GA_TIMED_OCC=2|4|8 selects, default 8 (full occupancy)
+inline int occupancy_target() {
+    static int v = [] { const char* e = getenv("GA_TIMED_OCC"); int x = e ? atoi(e) : 8; return (x == 2 || x == 4) ? x : 8; }();
+    return v;
+}
 inline uint32_t nblocks(uint32_t T, uint32_t block) { return (T + block - 1) / block; }
 inline ga_status launched() { return cudaGetLastError() == cudaSuccess ? GA_OK : GA_ECUDA; }
 
@@ -323,7 +330,12 @@ ga_status ga_trace_timed(ga_heap_t h, ga_stream_t stream, const uint32_t* sizes,
     if (!h || !sizes || !counts || T == 0 || D > 1) return GA_EINVAL;
     if (block == 0) block = 256;
     GaPolicy al{ga_dev_heap{h->ddesc, h->dev.base}};
-    k_timed<GaPolicy><<<nblocks(T, block), block, 0, (cudaStream_t)stream>>>(al, sizes, R, T, D, counts);
+    cudaStream_t s = (cudaStream_t)stream;
+    switch (occupancy_target()) {
+        case 2: k_timed<GaPolicy, 2><<<nblocks(T, block), block, 0, s>>>(al, sizes, R, T, D, counts); break;
+        case 4: k_timed<GaPolicy, 4><<<nblocks(T, block), block, 0, s>>>(al, sizes, R, T, D, counts); break;
+        default: k_timed<GaPolicy, 8><<<nblocks(T, block), block, 0, s>>>(al, sizes, R, T, D, counts); break;
+    }
     return launched();
 }
 
@@ -374,15 +386,17 @@ ga_status ga_cuda_trace_timed(ga_stream_t stream, const uint32_t* sizes, uint32_
                               uint64_t* counts, uint32_t block) {
     if (!sizes || !counts || T == 0 || D > 1) return GA_EINVAL;
     if (block == 0) block = 256;
-    k_timed<CudaPolicy><<<nblocks(T, block), block, 0, (cudaStream_t)stream>>>(CudaPolicy{}, sizes, R, T, D, counts);
+    k_timed<CudaPolicy, 8><<<nblocks(T, block), block, 0, (cudaStream_t)stream>>>(CudaPolicy{}, sizes, R, T, D, counts);
     return launched();
 }
 
 ga_status ga_kernel_info(int which, uint32_t block, int* regs, int* blocks_per_sm, int* local_bytes) {
     if (block == 0) block = 256;
     cudaFuncAttributes a;
-    const void* f = which == 0 ? (const void*)k_timed<GaPolicy> : which == 1 ? (const void*)k_churn_round<GaPolicy>
-                                                                              : (const void*)k_timed<CudaPolicy>;
+    int occ = occupancy_target();
+    const void* f = which == 0 ? (occ == 2 ? (const void*)k_timed<GaPolicy, 2> : occ == 4 ? (const void*)k_timed<GaPolicy, 4>
+                                                                                          : (const void*)k_timed<GaPolicy, 8>)
+                  : which == 1 ? (const void*)k_churn_round<GaPolicy> : (const void*)k_timed<CudaPolicy, 8>;
     if (cudaFuncGetAttributes(&a, f) != cudaSuccess) return GA_ECUDA;
     int nb = 0;
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, f, (int)block, 0) != cudaSuccess) return GA_ECUDA;

@@ -80,7 +80,10 @@ static __device__ __forceinline__ uint64_t a_exch(uint64_t* p, uint64_t v) { ret
 static __device__ __forceinline__ void red_add_release(uint64_t* p, uint64_t v) {
     asm volatile("red.release.gpu.global.add.u64 [%0], %1;" :: "l"(p), "l"(v) : "memory");
 }
-static __device__ __forceinline__ void fence() { __threadfence(); }
+// fence(): release/acquire ordering of our own accesses (publication paths);
+// fence_sc(): store -> load ordering for the clear-then-recheck (Dekker) patterns
+static __device__ __forceinline__ void fence() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
+static __device__ __forceinline__ void fence_sc() { __threadfence(); }
 static __device__ __forceinline__ void stat_add(const ga_desc* h, int i, uint64_t v) { a_add(&h->stats[i], v); }
 
 static __device__ __forceinline__ uint32_t hash32(uint32_t x) {
@@ -132,6 +135,11 @@ static __device__ __forceinline__ int32_t sem_D(uint64_t w) { return (int32_t)((
 static __device__ __forceinline__ void bsem_signal(uint64_t* s, uint32_t N, uint32_t B) {
     red_add_release(s, ((uint64_t)N << 32) - (uint64_t)B);
 }
+// signal after atomics whose returned values were already consumed (so they
+// have performed at L2): no release fence needed
+static __device__ __forceinline__ void bsem_signal_after_rmw(uint64_t* s, uint32_t N) {
+    asm volatile("red.relaxed.gpu.global.add.u64 [%0], %1;" :: "l"(s), "l"((uint64_t)N << 32) : "memory");
+}
 
 // try-wait (R-7): C -= N iff C >= N.  One fetch-add: subtract,
 // and give the units back if the pre-image was short.
@@ -139,7 +147,7 @@ static __device__ __forceinline__ bool bsem_trywait(uint64_t* s, uint32_t N) {
     if (sem_C(ld_rlx(s)) < (int32_t)N) return false;
     const uint64_t dn = (uint64_t)N << 32;
     uint64_t old = a_add(s, (uint64_t)0 - dn);
-    if (sem_C(old) >= (int32_t)N) { fence(); return true; }
+    if (sem_C(old) >= (int32_t)N) return true;
     a_add(s, dn);
     return false;
 }
@@ -162,10 +170,9 @@ static __device__ __noinline__ int bsem_wait(uint64_t* s, uint32_t N, uint32_t B
     for (;;) {
         uint64_t old = a_add(s, (uint64_t)0 - dn);
         int32_t C = sem_C(old), D = sem_D(old);
-        if (C >= (int32_t)N) { fence(); return kAcquired; }
+        if (C >= (int32_t)N) return kAcquired;
         if ((int64_t)C + D < (int64_t)N) {
             a_add(s, dn + (uint64_t)(B - N));                                   // C += N, E += B - N
-            fence();
             return kGrow;
         }
         uint64_t w = a_add(s, dn - (uint64_t)N) + dn - (uint64_t)N;            // C += N, R += N
@@ -209,7 +216,6 @@ __host__ __device__ inline uint32_t hb_total_words(uint32_t n0) {
 // propagate "word j of level k became non-zero" upwards
 static __device__ __forceinline__ void hb_up_set(const HB& b, int k, uint32_t j) {
     for (; k + 1 < b.nl; k++) {
-        fence();
         uint64_t old = a_or(&b.w[b.off[k + 1] + (j >> 6)], 1ull << (j & 63));
         if (old) return;
         j >>= 6;
@@ -221,7 +227,7 @@ static __device__ __noinline__ void hb_up_clear(const HB& b, int k, uint32_t j) 
         uint64_t* sw = &b.w[b.off[k + 1] + (j >> 6)];
         uint64_t bit = 1ull << (j & 63);
         uint64_t old = a_and(sw, ~bit);
-        fence();
+        fence_sc();
         if (ld_rlx(&b.w[b.off[k] + j]) != 0) {          // re-set: a setter raced with us
             uint64_t o2 = a_or(sw, bit);
             if (o2 == 0) hb_up_set(b, k + 1, j >> 6);
@@ -412,7 +418,6 @@ static __device__ __noinline__ uint64_t page_claim(const ga_desc* h, uint32_t A,
                     uint64_t old = a_or(&h->chunk_used[ch], m);
                     uint64_t got = m & ~old;
                     if (got) {
-                        fence();
                         if (ld_rlx32(&h->chunk_owner[ch]) != A + 1) {   // recycled chunk: undo
                             a_and(&h->chunk_used[ch], ~got);
                             break;
@@ -488,7 +493,7 @@ static __device__ __noinline__ void nonfull_clear_if_full(const ga_desc* h, uint
     uint64_t* nf = &h->chunk_nonfull[(p >> kChunkShift) * kNcls + c];
     uint64_t bit = 1ull << (p & (kChunkPages - 1));
     a_and(nf, ~bit);
-    fence();
+    fence_sc();
     uint64_t w[4];
     ld_bitmap(page_bits(h, p), w);
     if (ld_rlx32(&h->kind[p]) == kind_bin(A, c) && !page_full(w, c)) a_or(nf, bit);
@@ -508,7 +513,6 @@ static __device__ __noinline__ uint64_t bin_claim_page(const ga_desc* h, uint64_
             uint64_t old = a_or(&bw[i], m);
             uint64_t got = m & ~old;
             if (got) {
-                fence();
                 if (ld_rlx32(&h->kind[p]) != kind_bin(A, c)) {     // recycled page: undo as a free
                     a_and(&bw[i], ~got);
                     return 0;
@@ -592,7 +596,7 @@ static __device__ __forceinline__ void mark_candidate(const ga_desc* h, uint64_t
     uint64_t* cw = &h->chunk_cand[p >> kChunkShift];
     uint64_t bit = 1ull << (p & (kChunkPages - 1));
     if (!(ld_rlx(cw) & bit)) a_or(cw, bit);
-    fence();
+    fence_sc();
     if (!ld_rlx(&h->cand_any[A * kSemStride])) a_or(&h->cand_any[A * kSemStride], 1);
 }
 
@@ -601,7 +605,7 @@ static __device__ __noinline__ void reclaim_arena(const ga_desc* h, uint32_t A, 
     uint64_t* any = &h->cand_any[A * kSemStride];
     if (!ld_rlx(any)) return;
     a_exch(any, 0);
-    fence();
+    fence_sc();
     HB ob = owned_hb(h, A);
     bool left = false;
     for (uint32_t j = 0; j < ob.n[0]; j++) {
@@ -1019,7 +1023,7 @@ static __device__ __noinline__ void ga_free_off(const ga_desc* h, uint64_t off) 
     __syncwarp(bins);
     uint32_t key2 = (A << 3) | (uint32_t)c;
     unsigned g2 = __match_any_sync(bins, key2);
-    if ((int)lane_id() == __ffs(g2) - 1) bsem_signal(sem_ptr(h, A, c), __popc(g2), 0);
+    if ((int)lane_id() == __ffs(g2) - 1) bsem_signal_after_rmw(sem_ptr(h, A, c), __popc(g2));
 }
 
 }  // namespace ga
