@@ -152,40 +152,79 @@ static __device__ __forceinline__ bool bsem_trywait(uint64_t* s, uint32_t N) {
     return false;
 }
 
-// Alg. 1 (P:L650-672).  Returns kAcquired (0) or kGrow (-1; the caller must
-// produce B units, keep N and signal(B - N, B - N), or signal(0, B - N) on
-// failure, P:L756-764).  While blocked it runs `spin()` -- the delegated work
-// of Sec. 4.2.1 -- between polls.  Reading R-2: keep waiting while
-// C < N and R <= C + E, i.e. C < N and C + D >= 0.
-template <class Spin>
-static __device__ __noinline__ int bsem_wait(uint64_t* s, uint32_t N, uint32_t B, Spin spin) {
-    // Optimistic form of Alg. 1: one fetch-add C -= N decides on the pre-image.
-    //   pre C >= N           -> ACQUIRED (the common case: one atomic, no retry)
+// Alg. 1 core (documentation at bsem_wait below).
+template <bool kExact, class Spin>
+static __device__ __noinline__ int bsem_wait_impl(uint64_t* s, uint32_t N, uint32_t B, Spin spin) {
+    const uint64_t dn = (uint64_t)N << 32;
+    uint64_t w;
+    if (kExact) {
+        // Fast path: a plain load says the units are there -> one fetch-add.
+        // If it raced (pre-image short), give them back and run the exact form.
+        w = ld_rlx(s);
+        if (sem_C(w) >= (int32_t)N) {
+            uint64_t old = a_add(s, (uint64_t)0 - dn);
+            if (sem_C(old) >= (int32_t)N) return kAcquired;
+            w = a_add(s, dn) + dn;
+        }
+        // Exact Alg. 1: one CAS decides among the three branches on the current word.
+        for (;;) {
+            int32_t C = sem_C(w), D = sem_D(w);
+            uint64_t nw;
+            int res;
+            if ((int64_t)C + D < (int64_t)N) { nw = w + (uint64_t)(B - N); res = kGrow; }         // E += B - N
+            else if (C >= (int32_t)N) { nw = w - dn; res = kAcquired; }                        // C -= N
+            else { nw = w - (uint64_t)N; res = kBlocked; }                                      // R += N
+            uint64_t old = a_cas(s, w, nw);
+            if (old != w) { w = old; continue; }
+            if (res != kBlocked) return res;
+            uint32_t ns = 64;
+            for (;;) {                                                                          // R-2
+                w = ld_rlx(s);
+                if (!(sem_C(w) < (int32_t)N && (int64_t)sem_C(w) + sem_D(w) >= 0)) break;
+                spin();
+                __nanosleep(ns);
+                if (ns < 2048) ns <<= 1;
+            }
+            w = a_add(s, (uint64_t)N) + (uint64_t)N;                                            // R -= N
+        }
+    }
+    // Optimistic form: one fetch-add C -= N decides on the pre-image.
+    //   pre C >= N           -> ACQUIRED (one atomic, no retry)
     //   pre C + D < N        -> GROW: give C back, E += B - N
     //   otherwise            -> reserve: give C back, R += N (C + D unchanged), spin
-    // The conversion adds keep C + D exact for reservations; an in-flight GROW
-    // conversion hides its B units for one round trip (others may over-produce,
-    // never over-grant).  DESIGN.md "Semaphore word" and tests/test_fa_model.py.
-    const uint64_t dn = (uint64_t)N << 32;
+    // Reservation conversions keep C + D exact; an in-flight GROW conversion hides
+    // its units for one round trip, so others may over-produce (never over-grant).
     for (;;) {
         uint64_t old = a_add(s, (uint64_t)0 - dn);
         int32_t C = sem_C(old), D = sem_D(old);
         if (C >= (int32_t)N) return kAcquired;
         if ((int64_t)C + D < (int64_t)N) {
-            a_add(s, dn + (uint64_t)(B - N));                                   // C += N, E += B - N
+            a_add(s, dn + (uint64_t)(B - N));                                                   // C += N, E += B - N
             return kGrow;
         }
-        uint64_t w = a_add(s, dn - (uint64_t)N) + dn - (uint64_t)N;            // C += N, R += N
+        w = a_add(s, dn - (uint64_t)N) + dn - (uint64_t)N;                                     // C += N, R += N
         uint32_t ns = 64;
-        while (sem_C(w) < (int32_t)N && (int64_t)sem_C(w) + sem_D(w) >= 0) {    // R-2
+        while (sem_C(w) < (int32_t)N && (int64_t)sem_C(w) + sem_D(w) >= 0) {                    // R-2
             spin();
             __nanosleep(ns);
             if (ns < 2048) ns <<= 1;
             w = ld_rlx(s);
         }
-        a_add(s, (uint64_t)N);                                                  // R -= N
+        a_add(s, (uint64_t)N);                                                                  // R -= N
     }
 }
+// Alg. 1 (P:L650-672).  Returns kAcquired (0) or kGrow (-1; the caller must
+// produce B units, keep N and signal(B - N, B - N), or signal(0, B - N) on
+// failure, P:L756-764).  While blocked it runs `spin()` -- the delegated work
+// of Sec. 4.2.1 -- between polls.  Reading R-2: keep waiting while
+// C < N and R <= C + E, i.e. C < N and C + D >= 0.
+// bsem_wait: exact growth decisions (arena class / page semaphores: an extra
+//   batch costs real pages); bsem_wait_fast: optimistic (TBuddy orders: an extra
+//   split stays available inside the tree).  DESIGN.md "Semaphore word".
+template <class Spin>
+static __device__ __forceinline__ int bsem_wait(uint64_t* s, uint32_t N, uint32_t B, Spin spin) { return bsem_wait_impl<true>(s, N, B, spin); }
+template <class Spin>
+static __device__ __forceinline__ int bsem_wait_fast(uint64_t* s, uint32_t N, uint32_t B, Spin spin) { return bsem_wait_impl<false>(s, N, B, spin); }
 struct NoSpin { __device__ void operator()() const {} };
 
 // ---------------------------------------------------------------------------
@@ -323,7 +362,7 @@ static __device__ __noinline__ int64_t tree_alloc_one(const ga_desc* h, int o) {
             for (int k = o; k < m; k++) bsem_signal(tsem_ptr(h, k), 0, 1);
             return -1;
         }
-        if (bsem_wait(tsem_ptr(h, m), 1, 2, NoSpin()) == kAcquired) break;   // batch size two
+        if (bsem_wait_fast(tsem_ptr(h, m), 1, 2, NoSpin()) == kAcquired) break;   // batch size two
         m++;
     }
     uint64_t wj;
@@ -874,7 +913,7 @@ static __device__ __noinline__ Grant tree_leader_step(const ga_desc* h, TreeLead
                 g.kind = 4;
                 return g;
             }
-            int r = bsem_wait(tsem_ptr(h, m), Nk, 2 * ceil_half(Nk), NoSpin());
+            int r = bsem_wait_fast(tsem_ptr(h, m), Nk, 2 * ceil_half(Nk), NoSpin());
             if (r == kAcquired) break;
             Nk = ceil_half(Nk);
             m++;
