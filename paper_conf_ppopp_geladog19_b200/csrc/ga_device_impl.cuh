@@ -410,6 +410,21 @@ static __device__ __noinline__ void tree_free(const ga_desc* h, int n, uint64_t 
     }
 }
 
+// Does any order >= o show a unit (C >= 1) or growth / reservations in flight
+// (D != 0)?  At true exhaustion every such word is (0, 0).
+static __device__ __noinline__ bool tree_has_supply(const ga_desc* h, int o) {
+    for (int k = o; k <= (int)h->L; k++) {
+        uint64_t w = ld_rlx(tsem_ptr(h, k));
+        if (sem_C(w) >= 1 || sem_D(w) != 0) return true;
+    }
+    return false;
+}
+// Per-lane TBuddy allocation with the no-false-starvation retry: the optimistic
+// order semaphores can send a lane up the tree while another lane's split is
+// still being published (R-27 analogue).  Retry while the tree shows supply;
+// before giving up, drain deferred reclamation once (empty chunks go back).
+static __device__ __noinline__ int64_t tree_alloc_one_retry(const ga_desc* h, int o);
+
 // ---------------------------------------------------------------------------
 // 5. UAlloc: chunks, pages, bins
 // ---------------------------------------------------------------------------
@@ -670,6 +685,23 @@ static __device__ __noinline__ void reclaim_arena(const ga_desc* h, uint32_t A, 
 }
 static __device__ __noinline__ void reclaim_all(const ga_desc* h) {
     for (uint32_t A = 0; A < h->n_arenas; A++) reclaim_arena(h, A, -1);
+}
+
+static __device__ __noinline__ int64_t tree_alloc_one_retry(const ga_desc* h, int o) {
+    bool drained = false;
+    uint32_t ns = 64;
+    for (int attempt = 0; attempt < 256; attempt++) {
+        int64_t x = tree_alloc_one(h, o);
+        if (x >= 0) return x;
+        if (!tree_has_supply(h, o)) {
+            if (drained) return -1;
+            reclaim_all(h);
+            drained = true;
+            continue;
+        }
+        __nanosleep(ns); if (ns < 4096) ns <<= 1;
+    }
+    return -1;
 }
 
 // ---------------------------------------------------------------------------
@@ -975,11 +1007,7 @@ static __device__ __forceinline__ uint64_t group_malloc(const ga_desc* h, unsign
                     if (is_bin) my = bin_malloc_lane(h, arena_of(h), key);
                     else {
                         int o = key - kNcls;
-                        int64_t x = tree_alloc_one(h, o);
-                        if (x < 0) {
-                            reclaim_all(h);
-                            x = tree_alloc_one(h, o);
-                        }
+                        int64_t x = tree_alloc_one_retry(h, o);
                         if (x >= 0) {
                             uint64_t pg = (uint64_t)x << o;
                             st_rlx32(&h->kind[pg], kKindTree | (uint32_t)o);
