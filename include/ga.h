@@ -62,14 +62,16 @@ typedef struct ga_desc {
     uint64_t* sem;            /* [n_arenas][8] class bulk semaphores, 32 B apart        */
     uint64_t* psem;           /* [n_arenas] page bulk semaphores, 32 B apart            */
     uint32_t* hint;           /* [n_arenas][8] current bin page per class               */
-    uint64_t* owned;          /* [n_arenas] 2-level bitmaps of owned chunks             */
-    uint64_t* cand_any;       /* [n_arenas] nonzero when the arena has candidates       */
-    uint64_t* avail;          /* TBuddy availability bitmaps, all levels                */
+    uint64_t* ahb;            /* [n_arenas][10] chunk summaries (3-level bitsets): chunks
+                                 with free pages, with reclaim candidates, with non-full
+                                 bins of class c (c = 0..7)                             */
+    uint64_t* avail;          /* TBuddy availability bitmaps, all levels (3-level each)  */
     uint64_t* tsem;           /* [L+1] per-order bulk semaphores, 32 B apart            */
     uint64_t* stats;          /* device counters, see ga_stats_t                        */
-    uint64_t lvl_off[48];     /* word offset of level n (bits, then summaries)          */
-    uint32_t lvl_words[48];   /* words of level n's bitmap                              */
-    uint32_t lvl_sum1[48];    /* words of level n's first summary                       */
+    uint32_t ahb_words;       /* u64 words of one chunk summary                          */
+    uint32_t pad0;
+    uint64_t lvl_off[48];     /* word offset of level n in avail                        */
+    uint32_t lvl_words[48];   /* u64 words of level n's availability bits               */
 } ga_desc;
 
 /* Plain-old-data handle passed BY VALUE to kernels that call ga_malloc /

@@ -7,19 +7,19 @@
 // Sections:
 //   1. constants, PTX helpers
 //   2. bulk semaphore (Alg. 1 / Alg. 2) packed as (C, D = E - R) in
-//      one 64-bit word (reading R-6); wait is one CAS per attempt, signal one
-//      red.release.add
-//   3. hierarchical bitsets (find-any-set with scattered starts)
+//      one 64-bit word (reading R-6): a load-gated fetch-add fast path, the exact
+//      CAS form for arena semaphores, an optimistic form for TBuddy orders
+//   3. three-level summary bitsets (scattered search starts)
 //   4. TBuddy over per-level availability bitmaps; lock-free merge
 //      via a CAS on the word holding both siblings (reading R-21)
 //   5. UAlloc: per-SM arenas, 64-page chunks, one-page bins with
-//      out-of-band 256-bit slot bitmaps, per-class bulk semaphores
+//      out-of-band 256-bit slot bitmaps, per-(arena, class) chunk summaries
 //   6. deferred reclamation delegated to waiting threads
 //   7. warp-collective front end: __match_any_sync groups a warp's lanes by size
-//      class; one leader performs the semaphore operation and the bitmap claim
-//      for the whole group (collective critical section)
+//      class; one semaphore operation serves the group; the group claims its
+//      slots collectively, one atomicOr per bitmap word
 //
-// Invariants the code relies on:
+// Invariants:
 //   * bits[p][*] == all ones whenever page p is not a live bin, so a stale
 //     claimer's atomicOr can never take a slot in a recycled page;
 //   * kind[p] is written only while bits[p] is all ones; claimers re-validate it;
@@ -230,120 +230,121 @@ struct NoSpin { __device__ void operator()() const {} };
 // ---------------------------------------------------------------------------
 // 3. hierarchical bitsets: level 0 holds the data bits, level k+1 has one bit per
 // non-zero word of level k.  Summary bits may be transiently stale in either
-// direction; finders tolerate false positives, callers that hold semaphore
-// units retry on a false negative (a setter is about to publish its bit).
 // ---------------------------------------------------------------------------
-struct HB {
-    uint64_t* w;          // level 0 at w[0], then the summaries
-    uint32_t n[4];        // words per level
-    uint32_t off[4];      // word offset of each level
-    int nl;               // number of levels
-};
-__host__ __device__ inline HB hb_make(uint64_t* base, uint32_t n0) {
-    HB b; b.w = base; b.nl = 0;
-    uint32_t n = n0 ? n0 : 1, o = 0;
-    for (;;) {
-        b.n[b.nl] = n; b.off[b.nl] = o; b.nl++; o += n;
-        if (n == 1 || b.nl == 4) break;
-        n = (n + 63) / 64;
-    }
-    return b;
+// 3. three-level summary bitsets ("HB3").  Layout [w0 | w1 | w2]: w0 holds the
+// bits, bit j of w1 says "w0 word j may be non-zero", bit j of w2 the same for
+// w1.  Summary bits may be stale in either direction for a moment: finders
+// skip zero words (false positive), and callers that hold semaphore units retry
+// on a false negative (a setter is about to publish).  Used for the TBuddy
+// availability levels and for the per-arena chunk summaries.
+// ---------------------------------------------------------------------------
+struct HB3 { uint64_t* w0; uint32_t n0; };
+static __host__ __device__ __forceinline__ uint32_t hb3_n1(uint32_t n0) { return (n0 + 63) / 64; }
+static __host__ __device__ __forceinline__ uint32_t hb3_n2(uint32_t n0) { return (hb3_n1(n0) + 63) / 64; }
+static __host__ __device__ __forceinline__ uint32_t hb3_words(uint32_t n0) { return n0 + hb3_n1(n0) + hb3_n2(n0); }
+static __device__ __forceinline__ uint64_t* hb3_w1(HB3 b) { return b.w0 + b.n0; }
+static __device__ __forceinline__ uint64_t* hb3_w2(HB3 b) { return b.w0 + b.n0 + hb3_n1(b.n0); }
+
+// w0 word j went from zero to non-zero: publish it in the summaries
+static __device__ __forceinline__ void hb3_up_set(HB3 b, uint32_t j) {
+    if (a_or(&hb3_w1(b)[j >> 6], 1ull << (j & 63)) == 0) a_or(&hb3_w2(b)[j >> 12], 1ull << ((j >> 6) & 63));
 }
-__host__ __device__ inline uint32_t hb_total_words(uint32_t n0) {
-    HB b = hb_make(nullptr, n0); return b.off[b.nl - 1] + b.n[b.nl - 1];
+// set bit i of w0
+static __device__ __forceinline__ void hb3_set(HB3 b, uint64_t i) {
+    if (a_or(&b.w0[i >> 6], 1ull << (i & 63)) == 0) hb3_up_set(b, (uint32_t)(i >> 6));
 }
-// propagate "word j of level k became non-zero" upwards
-static __device__ __forceinline__ void hb_up_set(const HB& b, int k, uint32_t j) {
-    for (; k + 1 < b.nl; k++) {
-        uint64_t old = a_or(&b.w[b.off[k + 1] + (j >> 6)], 1ull << (j & 63));
-        if (old) return;
-        j >>= 6;
-    }
+// w0 word j was seen zero: clear its summary bit, then re-check (clear-then-recheck)
+static __device__ __noinline__ void hb3_up_clear(HB3 b, uint32_t j) {
+    uint64_t* w1 = hb3_w1(b);
+    uint64_t bit = 1ull << (j & 63);
+    uint64_t old = a_and(&w1[j >> 6], ~bit);
+    fence_sc();
+    if (ld_rlx(&b.w0[j]) != 0) { if (a_or(&w1[j >> 6], bit) == 0) a_or(&hb3_w2(b)[j >> 12], 1ull << ((j >> 6) & 63)); return; }
+    if ((old & ~bit) != 0) return;
+    uint32_t j1 = j >> 6;
+    uint64_t* w2 = hb3_w2(b);
+    uint64_t bit2 = 1ull << (j1 & 63);
+    a_and(&w2[j1 >> 6], ~bit2);
+    fence_sc();
+    if (ld_rlx(&w1[j1]) != 0) a_or(&w2[j1 >> 6], bit2);
 }
-// propagate "word j of level k became zero" upwards, with clear-then-recheck
-static __device__ __noinline__ void hb_up_clear(const HB& b, int k, uint32_t j) {
-    for (; k + 1 < b.nl; k++) {
-        uint64_t* sw = &b.w[b.off[k + 1] + (j >> 6)];
-        uint64_t bit = 1ull << (j & 63);
-        uint64_t old = a_and(sw, ~bit);
-        fence_sc();
-        if (ld_rlx(&b.w[b.off[k] + j]) != 0) {          // re-set: a setter raced with us
-            uint64_t o2 = a_or(sw, bit);
-            if (o2 == 0) hb_up_set(b, k + 1, j >> 6);
-            return;
-        }
-        if ((old & ~bit) != 0) return;                   // summary word still non-zero
-        j >>= 6;
-    }
+// Bit i of w0 summarises an outside data word (*data).  Clear the bit when the
+// data says "empty", re-checking the data after the clear.
+static __device__ __noinline__ void hb3_clear_summarised(HB3 b, uint64_t i, const uint64_t* data, uint64_t empty_value) {
+    uint64_t bit = 1ull << (i & 63);
+    uint64_t old = a_and(&b.w0[i >> 6], ~bit);
+    fence_sc();
+    if (ld_rlx(data) != empty_value) { if (a_or(&b.w0[i >> 6], bit) == 0) hb3_up_set(b, (uint32_t)(i >> 6)); return; }
+    if (old == bit) hb3_up_clear(b, (uint32_t)(i >> 6));
 }
-// set bit i (level 0); returns the previous level-0 word
-static __device__ __forceinline__ uint64_t hb_set(const HB& b, uint64_t i) {
-    uint64_t old = a_or(&b.w[i >> 6], 1ull << (i & 63));
-    if (old == 0) hb_up_set(b, 0, (uint32_t)(i >> 6));
-    return old;
-}
-// called after an atomic made level-0 word j zero
-static __device__ __forceinline__ void hb_word_zeroed(const HB& b, uint32_t j) { if (b.nl > 1) hb_up_clear(b, 0, j); }
-// find a level-0 word that looks non-zero, starting the search at a scattered
-// position; returns its index or -1
-static __device__ __noinline__ int64_t hb_find(const HB& b, uint32_t seed) {
-    int top = b.nl - 1;
-    uint32_t nt = b.n[top];
-    for (uint32_t t = 0; t < nt; t++) {
-        uint32_t j = (seed + t) % nt;
-        uint64_t x = ld_rlx(&b.w[b.off[top] + j]);
-        // depth-first descent through candidate bits (at most 4 levels)
-        uint32_t idx[4]; uint64_t rem[4];
-        int k = top; idx[k] = j; rem[k] = x;
-        while (k <= top) {
-            if (rem[k] == 0) { k++; continue; }
-            if (k == 0) return (int64_t)idx[0];
-            uint32_t bit = first_from(rem[k], seed >> (5 * k));
-            rem[k] &= ~(1ull << bit);
-            uint32_t child = idx[k] * 64 + bit;
-            if (child >= b.n[k - 1]) continue;
-            uint64_t y = ld_rlx(&b.w[b.off[k - 1] + child]);
-            if (y == 0) continue;
-            k--; idx[k] = child; rem[k] = y;
-            if (k == 0) return (int64_t)child;
+// a w0 word that looks non-zero, searched from a scattered start; -1 if none
+static __device__ __noinline__ int64_t hb3_find(HB3 b, uint32_t seed) {
+    const uint32_t n1 = hb3_n1(b.n0), n2 = hb3_n2(b.n0);
+    const uint64_t* w1 = hb3_w1(b);
+    const uint64_t* w2 = hb3_w2(b);
+    for (uint32_t t = 0; t < n2; t++) {
+        uint32_t j2 = (seed + t) % n2;
+        uint64_t x2 = ld_rlx(&w2[j2]);
+        while (x2) {
+            uint32_t b2 = first_from(x2, seed);
+            x2 &= ~(1ull << b2);
+            uint32_t j1 = j2 * 64 + b2;
+            if (j1 >= n1) continue;
+            uint64_t x1 = ld_rlx(&w1[j1]);
+            while (x1) {
+                uint32_t b1 = first_from(x1, seed >> 6);
+                x1 &= ~(1ull << b1);
+                uint32_t j0 = j1 * 64 + b1;
+                if (j0 < b.n0 && ld_rlx(&b.w0[j0]) != 0) return (int64_t)j0;
+            }
         }
     }
     return -1;
 }
-static __device__ __forceinline__ HB level_hb(const ga_desc* h, int n) { HB b = hb_make(h->avail + h->lvl_off[n], h->lvl_words[n]); return b; }
-static __device__ __forceinline__ HB owned_hb(const ga_desc* h, uint32_t A) {
-    uint32_t tw = hb_total_words(h->chunk_words);
-    return hb_make(h->owned + (uint64_t)A * tw, h->chunk_words);
+static __device__ __forceinline__ bool hb3_any(HB3 b) {
+    const uint64_t* w2 = hb3_w2(b);
+    for (uint32_t j = 0, n2 = hb3_n2(b.n0); j < n2; j++) if (ld_rlx(&w2[j])) return true;
+    return false;
+}
+
+// per-arena chunk summaries: which chunks of arena A have free pages (FPC),
+// reclaim candidates (CND), non-full bins of class c (NFC + c)
+enum { kAhbFpc = 0, kAhbCnd = 1, kAhbNfc = 2, kAhbPerArena = 2 + kNcls };
+static __device__ __forceinline__ HB3 arena_hb(const ga_desc* h, uint32_t A, int which) {
+    HB3 b; b.n0 = h->chunk_words; b.w0 = h->ahb + ((uint64_t)A * kAhbPerArena + which) * h->ahb_words; return b;
+}
+static __device__ __forceinline__ HB3 level_hb(const ga_desc* h, int n) {
+    HB3 b; b.n0 = h->lvl_words[n]; b.w0 = h->avail + h->lvl_off[n]; return b;
 }
 
 // ---------------------------------------------------------------------------
-// 4. TBuddy
+// 4. TBuddy over per-level availability bitmaps: bit i of level n
+// set <=> node (n, i) is Available.  Partial/Busy are implied by
+// the bits below a node, so no parent state needs locking.
 // ---------------------------------------------------------------------------
 static __device__ __forceinline__ bool node_inside(const ga_desc* h, int n, uint64_t i) { return ((i + 1) << n) <= h->pages; }
 
-// make node i of level n available (a split's right child, a freed root)
+// make node i of level n available (a split's right child) and count it
 static __device__ __forceinline__ void tree_publish(const ga_desc* h, int n, uint64_t i, uint32_t expected) {
-    HB b = level_hb(h, n);
-    hb_set(b, i);
-    bsem_signal(tsem_ptr(h, n), 1, expected);            // C += 1 (and retire E if it was expected)
+    hb3_set(level_hb(h, n), i);
+    bsem_signal(tsem_ptr(h, n), 1, expected);            // C += 1, retire the expected unit
 }
 
-// claim up to `need` available nodes of level n (caller holds `need` units of
-// tsem[n]); claims from one word; returns the word index and the claimed mask
-static __device__ __noinline__ uint64_t tree_claim_word(const ga_desc* h, int n, int need, uint32_t seed, uint64_t* word_out) {
-    HB b = level_hb(h, n);
+// claim up to `need` available nodes of level n from one bitmap word (the
+// caller holds `need` units of tsem[n]); returns the claimed mask, word in *wj
+static __device__ __noinline__ uint64_t tree_claim_word(const ga_desc* h, int n, int need, uint32_t seed, uint64_t* wj) {
+    HB3 b = level_hb(h, n);
     uint32_t ns = 32;
     for (;;) {
-        int64_t j = hb_find(b, seed);
+        int64_t j = hb3_find(b, seed);
         if (j >= 0) {
-            uint64_t* wp = &b.w[j];
-            uint64_t x = ld_rlx(wp);
+            uint64_t x = ld_rlx(&b.w0[j]);
             while (x) {
                 uint64_t m = lowest_bits(x, need);
-                uint64_t old = a_and(wp, ~m);
+                uint64_t old = a_and(&b.w0[j], ~m);
                 uint64_t got = old & m;
-                if ((old & ~m) == 0 && old != 0) hb_word_zeroed(b, (uint32_t)j);
-                if (got) { *word_out = (uint64_t)j; return got; }
+                if (old != 0 && (old & ~m) == 0) hb3_up_clear(b, (uint32_t)j);
+                if (got) { *wj = (uint64_t)j; return got; }
                 x = old & ~m;
             }
         }
@@ -352,59 +353,55 @@ static __device__ __noinline__ uint64_t tree_claim_word(const ga_desc* h, int n,
     }
 }
 
-// Single-thread allocation of one order-o block, iterative:
-// climb while wait says GROW, claim at the first level that grants, split down.
-// Returns the node index at level o, or -1 (every E retracted).
+// Single-thread allocation of one order-o block: climb while wait
+// says GROW, claim at the first level that grants, split down publishing the
+// right halves.  Returns the node at level o, or -1 (every E retracted).
 static __device__ __noinline__ int64_t tree_alloc_one(const ga_desc* h, int o) {
     int m = o;
     for (;;) {
-        if (m > (int)h->L) {                               // no parent: fail, retract E below
-            for (int k = o; k < m; k++) bsem_signal(tsem_ptr(h, k), 0, 1);
+        if (m > (int)h->L) {
+            for (int k = o; k < m; k++) bsem_signal(tsem_ptr(h, k), 0, 1);   // failure signal
             return -1;
         }
-        if (bsem_wait_fast(tsem_ptr(h, m), 1, 2, NoSpin()) == kAcquired) break;   // batch size two
+        if (bsem_wait_fast(tsem_ptr(h, m), 1, 2, NoSpin()) == kAcquired) break;   // batch two
         m++;
     }
     uint64_t wj;
     uint64_t got = tree_claim_word(h, m, 1, scatter_seed(), &wj);
     uint64_t x = wj * 64 + (uint64_t)(__ffsll((long long)got) - 1);
-    for (int k = m - 1; k >= o; k--) {                    // split: keep left, publish right
-        x = 2 * x;
-        tree_publish(h, k, x + 1, 1);
-    }
+    for (int k = m - 1; k >= o; k--) { x = 2 * x; tree_publish(h, k, x + 1, 1); }
     return (int64_t)x;
 }
 
 // Free node x of level n: merge with the buddy when try-wait and
-// the buddy's available->busy transition both succeed, cascading (R-19);
-// otherwise mark it available with one CAS on the word that holds both
+// the buddy's available->busy transition both succeed, cascading upwards
+// (R-19); otherwise mark x available with ONE CAS on the word holding both
 // siblings (R-21), so two siblings never both end up available.
 static __device__ __noinline__ void tree_free(const ga_desc* h, int n, uint64_t x) {
     uint32_t ns = 32;
     for (;;) {
-        HB b = level_hb(h, n);
-        uint64_t* wp = &b.w[x >> 6];
+        HB3 b = level_hb(h, n);
+        uint64_t* wp = &b.w0[x >> 6];
         uint64_t xb = 1ull << (x & 63), yb = 1ull << ((x ^ 1) & 63);
         bool root = (n >= (int)h->L) || !node_inside(h, n, x ^ 1);
         uint64_t w = ld_rlx(wp);
         if (!root && (w & yb)) {
             if (bsem_trywait(tsem_ptr(h, n), 1)) {
                 uint64_t old = a_and(wp, ~yb);
-                if (old & yb) {                           // merged: free the parent at n + 1
-                    if ((old & ~yb) == 0) hb_word_zeroed(b, (uint32_t)(x >> 6));
-                    x >>= 1; n++;
-                    ns = 32;
+                if (old & yb) {                               // merged: free the parent at n + 1
+                    if (old == yb) hb3_up_clear(b, (uint32_t)(x >> 6));
+                    x >>= 1; n++; ns = 32;
                     continue;
                 }
-                bsem_signal(tsem_ptr(h, n), 1, 0);        // buddy claimed meanwhile: give back
+                bsem_signal(tsem_ptr(h, n), 1, 0);            // buddy claimed meanwhile: give back
             } else {
-                __nanosleep(ns); if (ns < 1024) ns <<= 1; // buddy's unit is held by a claimer
+                __nanosleep(ns); if (ns < 1024) ns <<= 1;     // the buddy's unit is held by a claimer
             }
             continue;
         }
         uint64_t old = a_cas(wp, w, w | xb);
-        if (old != w) continue;                           // the pair changed: re-evaluate
-        if (w == 0) hb_up_set(b, 0, (uint32_t)(x >> 6));
+        if (old != w) continue;                               // the pair changed: re-evaluate
+        if (w == 0) hb3_up_set(b, (uint32_t)(x >> 6));
         bsem_signal(tsem_ptr(h, n), 1, 0);
         return;
     }
@@ -419,143 +416,143 @@ static __device__ __noinline__ bool tree_has_supply(const ga_desc* h, int o) {
     }
     return false;
 }
-// Per-lane TBuddy allocation with the no-false-starvation retry: the optimistic
-// order semaphores can send a lane up the tree while another lane's split is
-// still being published (R-27 analogue).  Retry while the tree shows supply;
-// before giving up, drain deferred reclamation once (empty chunks go back).
-static __device__ __noinline__ int64_t tree_alloc_one_retry(const ga_desc* h, int o);
 
 // ---------------------------------------------------------------------------
-// 5. UAlloc: chunks, pages, bins
+// 5. UAlloc: chunks of 64 pages owned by one arena, one-page bins
 // ---------------------------------------------------------------------------
 static __device__ __forceinline__ uint32_t kind_bin(uint32_t A, int c) { return kKindBin | (A << 8) | (uint32_t)c; }
+static __device__ __forceinline__ uint64_t* nonfull_word(const ga_desc* h, uint64_t ch, int c) { return &h->chunk_nonfull[ch * kNcls + c]; }
+static __device__ __forceinline__ bool page_full(const uint64_t w[4], int c) {
+    for (int i = 0; i < words_of(c); i++) if ((w[i] | ~valid_mask(c, i)) != ~0ull) return false;
+    return true;
+}
 
-// Reclamation (section 6) forward declarations
 static __device__ void reclaim_arena(const ga_desc* h, uint32_t A, int budget);
+// delegated work run by threads blocked in an arena semaphore wait (Sec. 4.2.1)
 struct ArenaSpin {
     const ga_desc* h; uint32_t A;
     __device__ void operator()() const { reclaim_arena(h, A, 4); }
 };
 
-// Take a new chunk from TBuddy for arena A, keep the first k pages, open the
-// rest.  Returns the chunk index or -1.
+// page p (class c, arena A) has a free slot again
+static __device__ __forceinline__ void nonfull_set(const ga_desc* h, uint64_t p, int c, uint32_t A) {
+    uint64_t* nf = nonfull_word(h, p >> kChunkShift, c);
+    uint64_t bit = 1ull << (p & (kChunkPages - 1));
+    if (ld_rlx(nf) & bit) return;
+    if (a_or(nf, bit) == 0) hb3_set(arena_hb(h, A, kAhbNfc + c), p >> kChunkShift);
+}
+// drop p from the non-full set if it is really full (clear-then-recheck)
+static __device__ __noinline__ void nonfull_clear_if_full(const ga_desc* h, uint64_t p, int c, uint32_t A) {
+    uint64_t ch = p >> kChunkShift;
+    uint64_t* nf = nonfull_word(h, ch, c);
+    uint64_t bit = 1ull << (p & (kChunkPages - 1));
+    uint64_t old = a_and(nf, ~bit);
+    fence_sc();
+    uint64_t w[4];
+    ld_bitmap(page_bits(h, p), w);
+    if (ld_rlx32(&h->kind[p]) == kind_bin(A, c) && !page_full(w, c)) {
+        if (a_or(nf, bit) == 0) hb3_set(arena_hb(h, A, kAhbNfc + c), ch);
+        return;
+    }
+    if (old == bit) hb3_clear_summarised(arena_hb(h, A, kAhbNfc + c), ch, nf, 0);
+}
+
+// Take a new chunk from TBuddy for arena A, keep its first k pages, open the rest.
 static __device__ __noinline__ int64_t chunk_acquire(const ga_desc* h, uint32_t A, uint32_t k) {
     int64_t ch = tree_alloc_one(h, kChunkOrder);
     if (ch < 0) return -1;
     st_rlx32(&h->chunk_owner[ch], A + 1);
     fence();
-    hb_set(owned_hb(h, A), (uint64_t)ch);
     uint64_t keep = k >= 64 ? ~0ull : ((1ull << k) - 1);
-    a_and(&h->chunk_used[ch], keep);                       // open pages k..63
+    a_and(&h->chunk_used[ch], keep);                          // open pages k..63 (all ones while unowned)
+    if (k < 64) hb3_set(arena_hb(h, A, kAhbFpc), (uint64_t)ch);
     stat_add(h, kStatChunkGrow, 1);
     return ch;
 }
 
-// Claim up to `need` free pages of one chunk owned by A (caller holds `need`
-// units of psem[A]).  Returns the mask of pages claimed, chunk in *ch_out.
+// Claim up to `need` free pages from ONE chunk of arena A (caller holds `need`
+// units of psem[A]): one atomicOr per attempt.  Returns the page mask, chunk in *ch_out.
 static __device__ __noinline__ uint64_t page_claim(const ga_desc* h, uint32_t A, int need, uint64_t* ch_out) {
-    HB ob = owned_hb(h, A);
+    HB3 fb = arena_hb(h, A, kAhbFpc);
     uint32_t seed = scatter_seed();
     uint32_t ns = 32;
     for (;;) {
-        // scan every owned chunk word
-        for (uint32_t t = 0; t < ob.n[0]; t++) {
-            uint32_t j = (seed + t) % ob.n[0];
-            uint64_t ow = ld_rlx(&ob.w[j]);
-            while (ow) {
-                uint32_t bit = (uint32_t)(__ffsll((long long)ow) - 1);
-                ow &= ow - 1;
+        int64_t j = hb3_find(fb, seed);
+        if (j >= 0) {
+            uint64_t cm = ld_rlx(&fb.w0[j]);
+            while (cm) {
+                uint32_t bit = first_from(cm, seed);
+                cm &= ~(1ull << bit);
                 uint64_t ch = (uint64_t)j * 64 + bit;
                 uint64_t u = ld_rlx(&h->chunk_used[ch]);
                 while (~u) {
                     uint64_t m = lowest_bits(~u, need);
                     uint64_t old = a_or(&h->chunk_used[ch], m);
                     uint64_t got = m & ~old;
-                    if (got) {
-                        if (ld_rlx32(&h->chunk_owner[ch]) != A + 1) {   // recycled chunk: undo
-                            a_and(&h->chunk_used[ch], ~got);
-                            break;
-                        }
-                        *ch_out = ch;
-                        return got;
-                    }
                     u = old | m;
+                    if (!got) continue;
+                    if (ld_rlx32(&h->chunk_owner[ch]) != A + 1) {  // recycled chunk: undo
+                        a_and(&h->chunk_used[ch], ~got);
+                        break;
+                    }
+                    if (u == ~0ull) hb3_clear_summarised(fb, ch, &h->chunk_used[ch], ~0ull);
+                    *ch_out = ch;
+                    return got;
                 }
+                if (u == ~0ull) hb3_clear_summarised(fb, ch, &h->chunk_used[ch], ~0ull);
             }
         }
         __nanosleep(ns); if (ns < 1024) ns <<= 1;
+        seed = hash32(seed + 5);
     }
 }
 
-// Return page p (chunk ch, owner A) to its chunk: C += 1 on psem[A].  An empty
-// chunk goes back to TBuddy (R-23).
 static __device__ void chunk_release(const ga_desc* h, uint64_t ch);
+// Return page p to its chunk (C += 1 on the owner's page semaphore); an empty
+// chunk goes back to TBuddy (R-23).
 static __device__ __noinline__ void page_release(const ga_desc* h, uint64_t p) {
     uint64_t ch = p >> kChunkShift;
     uint32_t A = ld_rlx32(&h->chunk_owner[ch]) - 1;
     uint64_t bit = 1ull << (p & (kChunkPages - 1));
     uint64_t old = a_and(&h->chunk_used[ch], ~bit);
+    if (old == ~0ull) hb3_set(arena_hb(h, A, kAhbFpc), ch);
     bsem_signal(psem_ptr(h, A), 1, 0);
     if ((old & ~bit) == 0) chunk_release(h, ch);
 }
 
-// An empty chunk back to the tree: try-wait all 64 page units, then take every
-// page with one CAS (0 -> all ones).  Failure leaves the chunk owned.
+// An empty chunk back to TBuddy: try-wait its 64 page units, then take every
+// page with one CAS (0 -> all ones).  Failure leaves the chunk with its arena.
 static __device__ __noinline__ void chunk_release(const ga_desc* h, uint64_t ch) {
     uint32_t A = ld_rlx32(&h->chunk_owner[ch]) - 1;
     if (A >= h->n_arenas) return;
     if (!bsem_trywait(psem_ptr(h, A), kChunkPages)) return;
     if (a_cas(&h->chunk_used[ch], 0ull, ~0ull) != 0ull) { bsem_signal(psem_ptr(h, A), kChunkPages, 0); return; }
-    HB ob = owned_hb(h, A);
-    uint64_t old = a_and(&ob.w[ch >> 6], ~(1ull << (ch & 63)));
-    if ((old & ~(1ull << (ch & 63))) == 0) hb_word_zeroed(ob, (uint32_t)(ch >> 6));
-    a_exch(&h->chunk_cand[ch], 0);
-    for (int c = 0; c < kNcls; c++) a_exch(&h->chunk_nonfull[ch * kNcls + c], 0);
+    hb3_clear_summarised(arena_hb(h, A, kAhbFpc), ch, &h->chunk_used[ch], ~0ull);
+    if (a_exch(&h->chunk_cand[ch], 0)) hb3_clear_summarised(arena_hb(h, A, kAhbCnd), ch, &h->chunk_cand[ch], 0);
     st_rlx32(&h->chunk_owner[ch], 0);
     fence();
     stat_add(h, kStatChunkReclaim, 1);
     tree_free(h, kChunkOrder, ch);
 }
 
-// Make page p a bin of class c for arena A.  The group keeps slots [0, take);
-// the others are opened (bitmap was all ones).  Returns true if slots remain.
-static __device__ __forceinline__ bool bin_init(const ga_desc* h, uint64_t p, uint32_t A, int c, uint32_t take) {
+// Make page p a bin of class c for arena A; the caller keeps slots [0, take),
+// the others are opened (the bitmap is all ones while p is not a bin).
+static __device__ __forceinline__ void bin_init(const ga_desc* h, uint64_t p, uint32_t A, int c, uint32_t take) {
     st_rlx32(&h->kind[p], kind_bin(A, c));
     fence();
     uint64_t* bw = page_bits(h, p);
     for (int w = 0; w < words_of(c); w++) {
-        uint64_t v = valid_mask(c, w);
-        int lo = (int)take - 64 * w;                      // kept slots in this word
+        int lo = (int)take - 64 * w;
         uint64_t keep = lo >= 64 ? ~0ull : lo <= 0 ? 0ull : ((1ull << lo) - 1);
-        uint64_t open = v & ~keep;
+        uint64_t open = valid_mask(c, w) & ~keep;
         if (open) a_and(&bw[w], ~open);
     }
-    return take < slots_of(c);
+    if (take < slots_of(c)) nonfull_set(h, p, c, A);
 }
 
-static __device__ __forceinline__ void nonfull_set(const ga_desc* h, uint64_t p, int c) {
-    uint64_t* nf = &h->chunk_nonfull[(p >> kChunkShift) * kNcls + c];
-    uint64_t bit = 1ull << (p & (kChunkPages - 1));
-    if (!(ld_rlx(nf) & bit)) a_or(nf, bit);
-}
-static __device__ __forceinline__ bool page_full(const uint64_t w[4], int c) {
-    for (int i = 0; i < words_of(c); i++) if ((w[i] | ~valid_mask(c, i)) != ~0ull) return false;
-    return true;
-}
-// clear-then-recheck: drop p from the nonfull set only if it is really full
-static __device__ __noinline__ void nonfull_clear_if_full(const ga_desc* h, uint64_t p, int c, uint32_t A) {
-    uint64_t* nf = &h->chunk_nonfull[(p >> kChunkShift) * kNcls + c];
-    uint64_t bit = 1ull << (p & (kChunkPages - 1));
-    a_and(nf, ~bit);
-    fence_sc();
-    uint64_t w[4];
-    ld_bitmap(page_bits(h, p), w);
-    if (ld_rlx32(&h->kind[p]) == kind_bin(A, c) && !page_full(w, c)) a_or(nf, bit);
-}
-
-// Try to claim up to `need` slots of page p (must be an (A, c) bin) from one
-// word.  Returns the claimed mask and word index; 0 if the page had none.
-static __device__ __noinline__ uint64_t bin_claim_page(const ga_desc* h, uint64_t p, uint32_t A, int c, int need, int* word_out) {
+// Claim up to `need` slots of page p (an (A, c) bin) from one bitmap word with
+// one atomicOr.  Returns the claimed mask (word in *wi); 0 if none.
+static __device__ __noinline__ uint64_t bin_claim_page(const ga_desc* h, uint64_t p, uint32_t A, int c, int need, int* wi) {
     if (ld_rlx32(&h->kind[p]) != kind_bin(A, c)) return 0;
     uint64_t* bw = page_bits(h, p);
     uint64_t w[4];
@@ -567,56 +564,66 @@ static __device__ __noinline__ uint64_t bin_claim_page(const ga_desc* h, uint64_
             uint64_t old = a_or(&bw[i], m);
             uint64_t got = m & ~old;
             if (got) {
-                if (ld_rlx32(&h->kind[p]) != kind_bin(A, c)) {     // recycled page: undo as a free
+                if (ld_rlx32(&h->kind[p]) != kind_bin(A, c)) {   // recycled page: undo
                     a_and(&bw[i], ~got);
                     return 0;
                 }
                 w[i] = old | m;
-                if ((w[i] | ~valid_mask(c, i)) == ~0ull) {       // this word is full now
+                if ((w[i] | ~valid_mask(c, i)) == ~0ull) {         // this word is full now
                     ld_bitmap(bw, w);
                     if (page_full(w, c)) nonfull_clear_if_full(h, p, c, A);
                 }
-                *word_out = i;
+                *wi = i;
                 return got;
             }
             fr = ~(old | m) & valid_mask(c, i);
         }
     }
+    nonfull_clear_if_full(h, p, c, A);
     return 0;
 }
 
-// Find a bin of (A, c) with a free slot: the arena hint first, then every
-// owned chunk's nonfull mask.  Returns the page or kNull.
-static __device__ __noinline__ uint64_t bin_find(const ga_desc* h, uint32_t A, int c, uint32_t seed) {
-    HB ob = owned_hb(h, A);
-    for (uint32_t t = 0; t < ob.n[0]; t++) {
-        uint32_t j = (seed + t) % ob.n[0];
-        uint64_t ow = ld_rlx(&ob.w[j]);
-        while (ow) {
-            uint32_t bit = (uint32_t)(__ffsll((long long)ow) - 1);
-            ow &= ow - 1;
-            uint64_t ch = (uint64_t)j * 64 + bit;
-            uint64_t nf = ld_rlx(&h->chunk_nonfull[ch * kNcls + c]);
-            while (nf) {
-                uint32_t pb = (uint32_t)(__ffsll((long long)nf) - 1);
-                nf &= nf - 1;
-                uint64_t p = ch * kChunkPages + pb;
-                uint64_t w[4];
-                ld_bitmap(page_bits(h, p), w);
-                if (ld_rlx32(&h->kind[p]) == kind_bin(A, c) && !page_full(w, c)) return p;
-                nonfull_clear_if_full(h, p, c, A);        // stale bit
+// A chunk of arena A with non-full class-c bins, and its non-full page mask:
+// the hint's chunk first, then the (A, c) summary.  Spins until one shows up
+// (the caller holds units, so a free slot exists or is being published).
+static __device__ __noinline__ uint64_t bin_find_chunk(const ga_desc* h, uint32_t A, int c, uint64_t* mask_out) {
+    uint32_t hp = ld_rlx32(&h->hint[A * kNcls + c]);
+    if (hp < h->pages) {
+        uint64_t m = ld_rlx(nonfull_word(h, hp >> kChunkShift, c));
+        if (m) { *mask_out = m; return hp >> kChunkShift; }
+    }
+    HB3 nb = arena_hb(h, A, kAhbNfc + c);
+    uint32_t seed = scatter_seed();
+    uint32_t ns = 32;
+    for (;;) {
+        int64_t j = hb3_find(nb, seed);
+        if (j >= 0) {
+            uint64_t cm = ld_rlx(&nb.w0[j]);
+            while (cm) {
+                uint32_t bit = first_from(cm, seed);
+                cm &= ~(1ull << bit);
+                uint64_t ch = (uint64_t)j * 64 + bit;
+                uint64_t m = ld_rlx(nonfull_word(h, ch, c));
+                if (m) {
+                    st_rlx32(&h->hint[A * kNcls + c], (uint32_t)(ch * kChunkPages + (__ffsll((long long)m) - 1)));
+                    *mask_out = m;
+                    return ch;
+                }
+                hb3_clear_summarised(nb, ch, nonfull_word(h, ch, c), 0);    // stale summary bit
             }
         }
+        __nanosleep(ns); if (ns < 1024) ns <<= 1;
+        seed = hash32(seed + 7);
     }
-    return kNull;
 }
 
 // ---------------------------------------------------------------------------
-// 6. deferred reclamation: frees that empty a bin only mark it;
-// threads blocked in a semaphore wait, growers and failing mallocs reclaim.
+// 6. deferred reclamation: a free that empties a bin only marks
+// it; threads blocked in a semaphore wait, growers about to take a new chunk,
+// failing mallocs and ga_heap_quiesce do the reclaiming.
 // ---------------------------------------------------------------------------
-// Reclaim page p if it is an empty bin: try-wait all its slots (R-22), then
-// take every slot word with a CAS (all free -> all ones).
+// Reclaim page p if it is an empty bin: try-wait all its slots (R-22), then take
+// every slot word with a CAS (all free -> all ones).
 static __device__ __noinline__ bool bin_reclaim(const ga_desc* h, uint64_t p) {
     uint32_t k = ld_rlx32(&h->kind[p]);
     if ((k & 0xC0000000u) != kKindBin) return false;
@@ -633,12 +640,15 @@ static __device__ __noinline__ bool bin_reclaim(const ga_desc* h, uint64_t p) {
         uint64_t v = valid_mask(c, i);
         if (a_cas(&bw[i], ~v, ~0ull) != ~v) break;
     }
-    if (i < words_of(c)) {                                // a slot was claimed meanwhile: undo
+    if (i < words_of(c)) {                                    // a slot was claimed meanwhile: undo
         for (int q = 0; q < i; q++) a_and(&bw[q], ~valid_mask(c, q));
         bsem_signal(sem_ptr(h, A, c), slots, 0);
         return false;
     }
-    a_and(&h->chunk_nonfull[(p >> kChunkShift) * kNcls + c], ~(1ull << (p & (kChunkPages - 1))));
+    uint64_t ch = p >> kChunkShift;
+    uint64_t* nf = nonfull_word(h, ch, c);
+    uint64_t bit = 1ull << (p & (kChunkPages - 1));
+    if (a_and(nf, ~bit) == bit) hb3_clear_summarised(arena_hb(h, A, kAhbNfc + c), ch, nf, 0);
     st_rlx32(&h->kind[p], 0);
     fence();
     stat_add(h, kStatBinReclaim, 1);
@@ -649,44 +659,39 @@ static __device__ __noinline__ bool bin_reclaim(const ga_desc* h, uint64_t p) {
 static __device__ __forceinline__ void mark_candidate(const ga_desc* h, uint64_t p, uint32_t A) {
     uint64_t* cw = &h->chunk_cand[p >> kChunkShift];
     uint64_t bit = 1ull << (p & (kChunkPages - 1));
-    if (!(ld_rlx(cw) & bit)) a_or(cw, bit);
-    fence_sc();
-    if (!ld_rlx(&h->cand_any[A * kSemStride])) a_or(&h->cand_any[A * kSemStride], 1);
+    if (ld_rlx(cw) & bit) return;
+    if (a_or(cw, bit) == 0) hb3_set(arena_hb(h, A, kAhbCnd), p >> kChunkShift);
 }
 
 // Reclaim up to `budget` candidate bins of arena A (budget < 0: all).
 static __device__ __noinline__ void reclaim_arena(const ga_desc* h, uint32_t A, int budget) {
-    uint64_t* any = &h->cand_any[A * kSemStride];
-    if (!ld_rlx(any)) return;
-    a_exch(any, 0);
-    fence_sc();
-    HB ob = owned_hb(h, A);
-    bool left = false;
-    for (uint32_t j = 0; j < ob.n[0]; j++) {
-        uint64_t ow = ld_rlx(&ob.w[j]);
-        while (ow) {
-            uint32_t bit = (uint32_t)(__ffsll((long long)ow) - 1);
-            ow &= ow - 1;
-            uint64_t ch = (uint64_t)j * 64 + bit;
-            if (!ld_rlx(&h->chunk_cand[ch])) continue;
-            if (budget == 0) { left = true; break; }
-            uint64_t cm = a_exch(&h->chunk_cand[ch], 0);
-            while (cm) {
-                uint32_t pb = (uint32_t)(__ffsll((long long)cm) - 1);
-                cm &= cm - 1;
-                if (budget == 0) { a_or(&h->chunk_cand[ch], 1ull << pb); left = true; continue; }
-                bin_reclaim(h, ch * kChunkPages + pb);
-                if (budget > 0) budget--;
-            }
+    HB3 cb = arena_hb(h, A, kAhbCnd);
+    if (!hb3_any(cb)) return;
+    uint32_t seed = scatter_seed();
+    while (budget != 0) {
+        int64_t j = hb3_find(cb, seed);
+        if (j < 0) return;
+        uint64_t cm = ld_rlx(&cb.w0[j]);
+        if (!cm) { hb3_up_clear(cb, (uint32_t)j); continue; }
+        uint64_t ch = (uint64_t)j * 64 + (uint64_t)(__ffsll((long long)cm) - 1);
+        uint64_t pm = a_exch(&h->chunk_cand[ch], 0);
+        hb3_clear_summarised(cb, ch, &h->chunk_cand[ch], 0);
+        while (pm) {
+            uint32_t pb = (uint32_t)(__ffsll((long long)pm) - 1);
+            pm &= pm - 1;
+            if (budget == 0) { mark_candidate(h, ch * kChunkPages + pb, A); continue; }
+            bin_reclaim(h, ch * kChunkPages + pb);
+            if (budget > 0) budget--;
         }
-        if (left) break;
     }
-    if (left) { fence(); a_or(any, 1); }
 }
 static __device__ __noinline__ void reclaim_all(const ga_desc* h) {
     for (uint32_t A = 0; A < h->n_arenas; A++) reclaim_arena(h, A, -1);
 }
 
+// Per-lane TBuddy allocation with the no-false-starvation retry: the optimistic
+// order semaphores can send a lane up the tree while another lane's split is
+// still in flight.  Retry while the tree shows supply; drain reclamation once.
 static __device__ __noinline__ int64_t tree_alloc_one_retry(const ga_desc* h, int o) {
     bool drained = false;
     uint32_t ns = 64;
@@ -705,173 +710,40 @@ static __device__ __noinline__ int64_t tree_alloc_one_retry(const ga_desc* h, in
 }
 
 // ---------------------------------------------------------------------------
-// 7. front end
+// 7. front end: warp-collective entry
 // ---------------------------------------------------------------------------
 // size -> key: 0..7 bin class, 8 + order for TBuddy, -1 for NULL
 static __device__ __forceinline__ int size_key(const ga_desc* h, uint64_t n) {
-    if (n == 0 || n > (h->pages << kPageShift)) return -1;                  // R-15
+    if (n == 0 || n > (h->pages << kPageShift)) return -1;             // R-15
     if (n <= 16) return 0;
-    int lg = 64 - __clzll((long long)(n - 1));                            // ceil(log2 n), R-14
-    if (lg <= 11) return lg - kMinShift;                                  // <= 2048 B: bins (R-12)
+    int lg = 64 - __clzll((long long)(n - 1));                         // ceil(log2 n), R-14
+    if (lg <= 11) return lg - kMinShift;                               // <= 2048 B: bins (R-12)
     int o = lg - kPageShift;
     if (o > (int)h->L) return -1;
     return kNcls + o;
 }
 
-// A grant tells the group which slots / nodes it received in one round.
-struct Grant {
-    uint64_t unit;      // bins: page; tree: word index at level m
-    uint64_t mask;      // bins: slot mask within word `word`; pages grant: page mask in chunk
-    uint32_t base;      // first group rank served
-    uint32_t count;     // ranks served
-    int word;           // bins: word of the page bitmap; tree: shift m - o
-    int kind;           // 0 slots, 1 fresh pages of a chunk, 2 tree nodes, 3 done, 4 failed
-};
-
-static __device__ __forceinline__ Grant shfl_grant(unsigned grp, Grant g, int src) {
-    Grant r;
-    r.unit = __shfl_sync(grp, g.unit, src);
-    r.mask = __shfl_sync(grp, g.mask, src);
-    r.base = __shfl_sync(grp, g.base, src);
-    r.count = __shfl_sync(grp, g.count, src);
-    r.word = __shfl_sync(grp, g.word, src);
-    r.kind = __shfl_sync(grp, g.kind, src);
-    return r;
+// Per-lane slow path (R-26, R-27): N = 1 waits; after local growth fails, drain
+// reclamation, then take pages and slots from other arenas before NULL.  Every
+// page source is tried before every other arena's bins (page sources only
+// shrink in malloc-only phases), so a malloc fails only if no arena can serve.
+static __device__ __noinline__ uint64_t bin_claim_one(const ga_desc* h, uint32_t A, int c) {
+    uint64_t csz = 16ull << c;
+    for (;;) {
+        uint64_t m;
+        uint64_t ch = bin_find_chunk(h, A, c, &m);
+        uint64_t p = ch * kChunkPages + (uint64_t)(__ffsll((long long)m) - 1);
+        int wi;
+        uint64_t got = bin_claim_page(h, p, A, c, 1, &wi);
+        if (got) return (p << kPageShift) + (uint64_t)(wi * 64 + __ffsll((long long)got) - 1) * csz;
+    }
 }
-
-// ---- bins, group path ------------------------------------------------------
-struct BinLeader {
-    uint32_t A; int c; uint32_t N;
-    uint32_t served;       // ranks served so far
-    int phase;             // 0 account, 1 claim existing, 2 fresh pages, 3 done
-    uint32_t pages_left;   // fresh pages still to track (phase 2)
-    uint32_t Bp;
-    uint64_t hint;
-    uint32_t seed;
-};
-
-static __device__ __noinline__ Grant bin_leader_step(const ga_desc* h, BinLeader& L) {
-    Grant g; g.kind = 3; g.base = L.served; g.count = 0; g.unit = 0; g.mask = 0; g.word = 0;
-    uint32_t slots = slots_of(L.c);
-    if (L.phase == 0) {
-        L.Bp = slots * ((L.N + slots - 1) / slots);                          // R-8
-        int r = bsem_wait(sem_ptr(h, L.A, L.c), L.N, L.Bp, ArenaSpin{h, L.A});
-        if (r == kAcquired) { L.phase = 1; L.hint = ld_rlx32(&h->hint[L.A * kNcls + L.c]); }
-        else {
-            // GROW: B'/slots new bins; pages accounted on the arena's page semaphore
-            uint32_t k = L.Bp / slots;
-            int rp = bsem_wait(psem_ptr(h, L.A), k, kChunkPages, ArenaSpin{h, L.A});
-            if (rp == kGrow) {
-                reclaim_arena(h, L.A, -1);                 // delegated work before a new chunk
-                int64_t ch = chunk_acquire(h, L.A, k);
-                if (ch < 0) {
-                    bsem_signal(psem_ptr(h, L.A), 0, kChunkPages - k);
-                    bsem_signal(sem_ptr(h, L.A, L.c), 0, L.Bp - L.N);
-                    g.kind = 4;
-                    return g;
-                }
-                bsem_signal(psem_ptr(h, L.A), kChunkPages - k, kChunkPages - k);
-                L.phase = 2; L.pages_left = 0;
-                // the whole batch sits in this chunk: pages 0..k-1
-                uint64_t pm = k >= 64 ? ~0ull : ((1ull << k) - 1);
-                uint32_t take_total = L.N;
-                for (uint32_t i = 0; i < k; i++) {
-                    uint32_t take = take_total > slots ? slots : take_total;
-                    take_total -= take;
-                    if (bin_init(h, (uint64_t)ch * kChunkPages + i, L.A, L.c, take))
-                        nonfull_set(h, (uint64_t)ch * kChunkPages + i, L.c);
-                }
-                stat_add(h, kStatBinGrow, k);
-                g.kind = 1; g.unit = (uint64_t)ch; g.mask = pm; g.count = L.N; g.word = (int)slots;
-                L.served = L.N;
-                L.hint = (uint64_t)ch * kChunkPages + k - 1;
-                st_rlx32(&h->hint[L.A * kNcls + L.c], (uint32_t)L.hint);
-                bsem_signal(sem_ptr(h, L.A, L.c), L.Bp - L.N, L.Bp - L.N);
-                L.phase = 3;
-                return g;
-            }
-            L.phase = 2; L.pages_left = k;
-        }
-    }
-    if (L.phase == 2) {
-        // track pages_left pages from the arena's chunks (units already held)
-        uint64_t ch;
-        uint64_t pm = page_claim(h, L.A, (int)L.pages_left, &ch);
-        uint32_t np = __popcll(pm);
-        uint32_t rem = L.N - L.served;
-        uint32_t serve = np * slots < rem ? np * slots : rem;
-        uint32_t left = serve;
-        for (uint32_t i = 0; i < np; i++) {
-            uint64_t p = ch * kChunkPages + nth_set(pm, i);
-            uint32_t take = left > slots ? slots : left;
-            left -= take;
-            if (bin_init(h, p, L.A, L.c, take)) nonfull_set(h, p, L.c);
-            L.hint = p;
-        }
-        stat_add(h, kStatBinGrow, np);
-        L.pages_left -= np;
-        g.kind = 1; g.unit = ch; g.mask = pm; g.count = serve; g.word = (int)slots;
-        L.served += serve;
-        if (L.pages_left == 0) {
-            st_rlx32(&h->hint[L.A * kNcls + L.c], (uint32_t)L.hint);
-            bsem_signal(sem_ptr(h, L.A, L.c), L.Bp - L.N, L.Bp - L.N);
-            L.phase = 3;
-        }
-        return g;
-    }
-    if (L.phase == 1) {
-        uint32_t ns = 32;
-        for (;;) {
-            uint64_t p = L.hint;
-            if (p < h->pages) {
-                int wi;
-                uint64_t got = bin_claim_page(h, p, L.A, L.c, (int)(L.N - L.served), &wi);
-                if (got) {
-                    uint32_t n = __popcll(got);
-                    g.kind = 0; g.unit = p; g.mask = got; g.word = wi; g.count = n;
-                    L.served += n;
-                    if (L.served == L.N) {
-                        L.phase = 3;
-                        if (ld_rlx32(&h->hint[L.A * kNcls + L.c]) != (uint32_t)p) st_rlx32(&h->hint[L.A * kNcls + L.c], (uint32_t)p);
-                    }
-                    return g;
-                }
-            }
-            uint64_t q = bin_find(h, L.A, L.c, L.seed);
-            if (q != kNull) { L.hint = q; continue; }
-            // units are held but no bin is visible yet: a free / grower is publishing
-            L.hint = kNull;
-            __nanosleep(ns); if (ns < 1024) ns <<= 1;
-            L.seed = hash32(L.seed + 7);
-        }
-    }
-    return g;
-}
-
-// Per-lane slow path (R-26, R-27): N = 1 waits; after local growth fails,
-// drain reclamation, then take pages and slots from other arenas before NULL.
 static __device__ __noinline__ uint64_t bin_malloc_lane(const ga_desc* h, uint32_t A0, int c) {
     uint32_t slots = slots_of(c);
-    uint64_t csz = 16ull << c;
     for (int attempt = 0; attempt < 2; attempt++) {
-        int r = bsem_wait(sem_ptr(h, A0, c), 1, slots, ArenaSpin{h, A0});
-        if (r == kAcquired) {
-            uint32_t seed = scatter_seed();
-            uint32_t ns = 32;
-            uint64_t p = ld_rlx32(&h->hint[A0 * kNcls + c]);
-            for (;;) {
-                if (p < h->pages) {
-                    int wi;
-                    uint64_t got = bin_claim_page(h, p, A0, c, 1, &wi);
-                    if (got) return (p << kPageShift) + (uint64_t)(wi * 64 + __ffsll((long long)got) - 1) * csz;
-                }
-                p = bin_find(h, A0, c, seed);
-                if (p == kNull) { __nanosleep(ns); if (ns < 1024) ns <<= 1; seed = hash32(seed + 3); }
-            }
-        }
-        int rp = bsem_wait(psem_ptr(h, A0), 1, kChunkPages, ArenaSpin{h, A0});
+        if (bsem_wait(sem_ptr(h, A0, c), 1, slots, ArenaSpin{h, A0}) == kAcquired) return bin_claim_one(h, A0, c);
         uint64_t p = kNull;
-        if (rp == kAcquired) {
+        if (bsem_wait(psem_ptr(h, A0), 1, kChunkPages, ArenaSpin{h, A0}) == kAcquired) {
             uint64_t ch;
             uint64_t pm = page_claim(h, A0, 1, &ch);
             p = ch * kChunkPages + (uint64_t)(__ffsll((long long)pm) - 1);
@@ -882,7 +754,7 @@ static __device__ __noinline__ uint64_t bin_malloc_lane(const ga_desc* h, uint32
             else bsem_signal(psem_ptr(h, A0), 0, kChunkPages - 1);
         }
         if (p != kNull) {
-            if (bin_init(h, p, A0, c, 1)) nonfull_set(h, p, c);
+            bin_init(h, p, A0, c, 1);
             stat_add(h, kStatBinGrow, 1);
             st_rlx32(&h->hint[A0 * kNcls + c], (uint32_t)p);
             bsem_signal(sem_ptr(h, A0, c), slots - 1, slots - 1);
@@ -891,16 +763,13 @@ static __device__ __noinline__ uint64_t bin_malloc_lane(const ga_desc* h, uint32
         bsem_signal(sem_ptr(h, A0, c), 0, slots - 1);
         if (attempt == 0) reclaim_all(h);
     }
-    // every page source first (they only shrink in malloc-only phases), then
-    // every arena's bins of this class: a malloc fails only if no arena can
-    // serve it (R-26)
     for (uint32_t t = 1; t <= h->n_arenas; t++) {
         uint32_t B = (A0 + t) % h->n_arenas;
         if (bsem_wait(psem_ptr(h, B), 1, 1, NoSpin()) == kAcquired) {
             uint64_t ch;
             uint64_t pm = page_claim(h, B, 1, &ch);
             uint64_t p = ch * kChunkPages + (uint64_t)(__ffsll((long long)pm) - 1);
-            if (bin_init(h, p, B, c, 1)) nonfull_set(h, p, c);
+            bin_init(h, p, B, c, 1);
             stat_add(h, kStatBinGrow, 1);
             bsem_signal(sem_ptr(h, B, c), slots - 1, 0);
             return p << kPageShift;
@@ -908,178 +777,255 @@ static __device__ __noinline__ uint64_t bin_malloc_lane(const ga_desc* h, uint32
     }
     for (uint32_t t = 1; t <= h->n_arenas; t++) {
         uint32_t B = (A0 + t) % h->n_arenas;
-        if (bsem_wait(sem_ptr(h, B, c), 1, 1, NoSpin()) == kAcquired) {
-            uint32_t seed = scatter_seed();
-            uint32_t ns = 32;
-            uint64_t p = ld_rlx32(&h->hint[B * kNcls + c]);
-            for (;;) {
-                if (p < h->pages) {
-                    int wi;
-                    uint64_t got = bin_claim_page(h, p, B, c, 1, &wi);
-                    if (got) return (p << kPageShift) + (uint64_t)(wi * 64 + __ffsll((long long)got) - 1) * csz;
-                }
-                p = bin_find(h, B, c, seed);
-                if (p == kNull) { __nanosleep(ns); if (ns < 1024) ns <<= 1; seed = hash32(seed + 3); }
-            }
-        }
+        if (bsem_wait(sem_ptr(h, B, c), 1, 1, NoSpin()) == kAcquired) return bin_claim_one(h, B, c);
     }
     stat_add(h, kStatFail, 1);
     return kNull;
 }
 
-// ---- TBuddy, group path ----------------------------------------------------
-struct TreeLeader {
-    int o; int m; uint32_t N; uint32_t Nm; uint32_t served; uint32_t seed; int phase;
-};
-static __device__ __forceinline__ uint32_t ceil_half(uint32_t x) { return (x + 1) >> 1; }
-
-static __device__ __noinline__ Grant tree_leader_step(const ga_desc* h, TreeLeader& L) {
-    Grant g; g.kind = 3; g.base = L.served; g.count = 0; g.unit = 0; g.mask = 0; g.word = 0;
-    if (L.phase == 0) {
-        uint32_t Nk = L.N;
-        int m = L.o;
-        for (;;) {
-            if (m > (int)h->L) {                              // nothing to grow from: retract E
-                uint32_t nk = L.N;
-                for (int k = L.o; k < m; k++) { bsem_signal(tsem_ptr(h, k), 0, 2 * ceil_half(nk) - nk); nk = ceil_half(nk); }
-                g.kind = 4;
-                return g;
-            }
-            int r = bsem_wait_fast(tsem_ptr(h, m), Nk, 2 * ceil_half(Nk), NoSpin());
-            if (r == kAcquired) break;
-            Nk = ceil_half(Nk);
-            m++;
-        }
-        L.m = m; L.Nm = Nk; L.phase = 1;
+// ---- bins: collective claim of one slot per lane (units already acquired) ----
+// Lanes spread over the chunk's non-full pages by their rank (each thread walks
+// the number of elements its index dictates), lanes that picked
+// the same page regroup and that page gets ONE atomicOr for all of them.
+static __device__ __noinline__ uint64_t bin_claim_collective(const ga_desc* h, unsigned grp, uint32_t A, int c) {
+    const uint32_t lane = lane_id();
+    const uint32_t per_page = slots_of(c) < 64 ? slots_of(c) : 64;
+    const uint64_t csz = 16ull << c;
+    uint64_t my = kNull;
+    unsigned unsat = grp;
+    while (unsat) {
+        const int L = __ffs(unsat) - 1;
+        uint64_t ch = 0, m = 0;
+        if ((int)lane == L) ch = bin_find_chunk(h, A, c, &m);
+        ch = __shfl_sync(unsat, ch, L);
+        m = __shfl_sync(unsat, m, L);
+        const uint32_t q = __popc(unsat & lanemask_lt());
+        const uint32_t np = __popcll(m);
+        const uint64_t page = ch * kChunkPages + nth_set(m, (q / per_page) % np);
+        const unsigned pg = __match_any_sync(unsat, page);
+        const int pl = __ffs(pg) - 1;
+        uint64_t got = 0;
+        int wi = 0;
+        if ((int)lane == pl) got = bin_claim_page(h, page, A, c, __popc(pg), &wi);
+        got = __shfl_sync(pg, got, pl);
+        wi = __shfl_sync(pg, wi, pl);
+        const uint32_t pr = __popc(pg & lanemask_lt());
+        if (pr < (uint32_t)__popcll(got)) my = (page << kPageShift) + (uint64_t)(wi * 64 + nth_set(got, pr)) * csz;
+        unsat = __ballot_sync(unsat, my == kNull);
     }
-    if (L.phase == 1) {
-        int s = L.m - L.o;
-        uint32_t need_nodes = L.Nm - ((L.served + (1u << s) - 1) >> s);
-        uint64_t wj;
-        uint64_t got = tree_claim_word(h, L.m, (int)need_nodes, L.seed, &wj);
-        uint32_t nn = __popcll(got);
-        uint32_t rem = L.N - L.served;
-        uint32_t cap = nn << s;
-        uint32_t serve = cap < rem ? cap : rem;
-        if (serve == rem && s > 0) {
-            // the last node is split: publish the unused right parts (E at each level)
-            uint64_t xlast = wj * 64 + (63 - __clzll((long long)got));
-            uint32_t keep_last = serve - ((nn - 1) << s);
-            uint64_t pos = keep_last;
-            for (int j = 0; j < s; j++) {
-                if ((pos >> j) & 1) {
-                    tree_publish(h, L.o + j, ((xlast << s) + pos) >> j, 1);
-                    pos += 1ull << j;
-                }
-            }
-        }
-        g.kind = 2; g.unit = wj; g.mask = got; g.count = serve; g.word = s;
-        L.served += serve;
-        if (L.served == L.N) L.phase = 3;
-        return g;
-    }
-    return g;
+    return my;
 }
 
-// ---- the group driver --------------------------------------------------------
-// Every lane of `grp` calls this with the same key; returns this lane's offset.
-static __device__ __forceinline__ uint64_t group_malloc(const ga_desc* h, unsigned grp, int key) {
-    const int lane = (int)lane_id();
+// ---- bins: collective growth (class semaphore said GROW for the group) ------
+// The leader accounts ceil(N/slots) pages on the arena page semaphore and
+// tracks them one chunk at a time (one atomicOr claims several pages: the
+// collective chunk-list split of P:L1282-1292); every lane computes its page
+// and slot, the first lane of each page initialises that bin, then the leader
+// publishes the spare slots with one signal.  Returns kNull for every lane if
+// the group could not grow (the caller degrades to per-lane waits).
+static __device__ __noinline__ uint64_t bin_grow_collective(const ga_desc* h, unsigned grp, uint32_t A, int c) {
+    const uint32_t lane = lane_id();
     const int leader = __ffs(grp) - 1;
-    const uint32_t N = __popc(grp);
-    const uint32_t rank = __popc(grp & lanemask_lt());
+    const uint32_t N = __popc(grp), rank = __popc(grp & lanemask_lt());
+    const uint32_t slots = slots_of(c);
+    const uint32_t Bp = slots * ((N + slots - 1) / slots);                 // R-8
+    const uint32_t k = Bp / slots;
+    const uint64_t csz = 16ull << c;
     uint64_t my = kNull;
-    BinLeader bl; TreeLeader tl;
-    bool is_bin = key < kNcls;
-    if (lane == leader) {
-        if (is_bin) { bl.A = arena_of(h); bl.c = key; bl.N = N; bl.served = 0; bl.phase = 0; bl.pages_left = 0; bl.Bp = 0; bl.hint = kNull; bl.seed = scatter_seed(); }
-        else { tl.o = key - kNcls; tl.m = tl.o; tl.N = N; tl.Nm = 0; tl.served = 0; tl.seed = scatter_seed(); tl.phase = 0; }
-    }
-    for (;;) {
-        Grant g;
-        if (lane == leader) g = is_bin ? bin_leader_step(h, bl) : tree_leader_step(h, tl);
-        g = shfl_grant(grp, g, leader);
-        if (g.kind >= 3) {
-            if (g.kind == 4) {
-                // R-27: the group could not be served as a whole -> per lane
-                if (lane == leader) stat_add(h, kStatFallback, 1);
-                if (my == kNull) {
-                    if (is_bin) my = bin_malloc_lane(h, arena_of(h), key);
-                    else {
-                        int o = key - kNcls;
-                        int64_t x = tree_alloc_one_retry(h, o);
-                        if (x >= 0) {
-                            uint64_t pg = (uint64_t)x << o;
-                            st_rlx32(&h->kind[pg], kKindTree | (uint32_t)o);
-                            my = pg << kPageShift;
-                        } else stat_add(h, kStatFail, 1);
-                    }
-                }
-            }
-            break;
-        }
-        if (rank >= g.base && rank < g.base + g.count) {
-            uint32_t r = rank - g.base;
-            if (g.kind == 0) {
-                uint32_t b = nth_set(g.mask, r);
-                my = (g.unit << kPageShift) + (uint64_t)(g.word * 64 + b) * (16ull << key);
-            } else if (g.kind == 1) {
-                uint32_t slots = (uint32_t)g.word;
-                uint64_t p = g.unit * kChunkPages + nth_set(g.mask, r / slots);
-                my = (p << kPageShift) + (uint64_t)(r % slots) * (16ull << key);
+    int mode = 0;                                                            // 0 claim pages, 1 fresh chunk, -1 fail
+    uint64_t ch = 0, pm = 0;
+    if ((int)lane == leader) {
+        if (bsem_wait(psem_ptr(h, A), k, kChunkPages, ArenaSpin{h, A}) == kGrow) {
+            reclaim_arena(h, A, -1);                                         // delegated work first
+            int64_t nc = chunk_acquire(h, A, k);
+            if (nc < 0) {
+                bsem_signal(psem_ptr(h, A), 0, kChunkPages - k);
+                bsem_signal(sem_ptr(h, A, c), 0, Bp - N);
+                mode = -1;
             } else {
-                int s = g.word, o = key - kNcls;
-                uint64_t x = g.unit * 64 + nth_set(g.mask, r >> s);
-                uint64_t node = (x << s) + (r & ((1u << s) - 1));
-                uint64_t pg = node << o;
+                bsem_signal(psem_ptr(h, A), kChunkPages - k, kChunkPages - k);
+                mode = 1; ch = (uint64_t)nc; pm = k >= 64 ? ~0ull : ((1ull << k) - 1);
+            }
+        }
+    }
+    mode = __shfl_sync(grp, mode, leader);
+    if (mode < 0) return kNull;
+    uint32_t served = 0, pages_left = k;
+    uint64_t last_page = 0;
+    while (pages_left) {
+        if (mode == 0 && (int)lane == leader) pm = page_claim(h, A, (int)pages_left, &ch);
+        ch = __shfl_sync(grp, ch, leader);
+        pm = __shfl_sync(grp, pm, leader);
+        const uint32_t np = __popcll(pm);
+        const uint32_t cap = np * slots;
+        if (rank >= served && rank < served + cap) {
+            const uint32_t r = rank - served;
+            const uint64_t p = ch * kChunkPages + nth_set(pm, r / slots);
+            my = (p << kPageShift) + (uint64_t)(r % slots) * csz;
+            if (r % slots == 0) {
+                const uint32_t left = N - served - (r / slots) * slots;
+                bin_init(h, p, A, c, left < slots ? left : slots);
+            }
+        }
+        last_page = ch * kChunkPages + nth_set(pm, np - 1);
+        served += cap < N - served ? cap : N - served;
+        pages_left -= np;
+        mode = 0;
+    }
+    __syncwarp(grp);
+    if ((int)lane == leader) {
+        stat_add(h, kStatBinGrow, k);
+        st_rlx32(&h->hint[A * kNcls + c], (uint32_t)last_page);
+        bsem_signal(sem_ptr(h, A, c), Bp - N, Bp - N);                      // release: bins are initialised
+    }
+    return my;
+}
+
+// ---- TBuddy, group path -------------------------------------------------------
+// One bulk wait of N units per order for the group (batch 2, B' = 2*ceil(N/2));
+// on GROW the group climbs with N_{k+1} = ceil(N_k / 2), claims N_m nodes at the
+// granting level m and splits them down: each claimed node serves 2^(m-o)
+// lanes, the unused right parts of the last node are published.  Returns kNull
+// for every lane if the tree could not serve the whole group.
+static __device__ __noinline__ uint64_t tree_malloc_group(const ga_desc* h, unsigned grp, int o) {
+    const uint32_t lane = lane_id();
+    const int leader = __ffs(grp) - 1;
+    const uint32_t N = __popc(grp), rank = __popc(grp & lanemask_lt());
+    int m = o;
+    uint32_t Nm = N;
+    if ((int)lane == leader) {
+        for (;;) {
+            if (m > (int)h->L) {
+                uint32_t nk = N;
+                for (int k = o; k < m; k++) { bsem_signal(tsem_ptr(h, k), 0, 2 * ((nk + 1) >> 1) - nk); nk = (nk + 1) >> 1; }
+                m = -1;
+                break;
+            }
+            if (bsem_wait_fast(tsem_ptr(h, m), Nm, 2 * ((Nm + 1) >> 1), NoSpin()) == kAcquired) break;
+            Nm = (Nm + 1) >> 1;
+            m++;
+        }
+    }
+    m = __shfl_sync(grp, m, leader);
+    if (m < 0) return kNull;
+    const int s = m - o;
+    uint64_t my = kNull;
+    uint32_t served = 0;
+    uint32_t seed = scatter_seed();
+    while (served < N) {
+        uint64_t wj = 0, got = 0;
+        if ((int)lane == leader) {
+            uint32_t need_nodes = Nm - (served >> s);
+            got = tree_claim_word(h, m, (int)need_nodes, seed, &wj);
+            uint32_t nn = __popcll(got);
+            uint32_t rem = N - served;
+            if ((nn << s) >= rem && s > 0) {
+                // the last node is split: publish its unused right parts (E at each level)
+                uint64_t xlast = wj * 64 + (63 - __clzll((long long)got));
+                uint64_t pos = rem - ((nn - 1) << s);
+                for (int j = 0; j < s; j++)
+                    if ((pos >> j) & 1) { tree_publish(h, o + j, ((xlast << s) + pos) >> j, 1); pos += 1ull << j; }
+            }
+        }
+        wj = __shfl_sync(grp, wj, leader);
+        got = __shfl_sync(grp, got, leader);
+        const uint32_t cap = (uint32_t)__popcll(got) << s;
+        if (rank >= served && rank < served + cap) {
+            const uint32_t r = rank - served;
+            const uint64_t x = wj * 64 + nth_set(got, r >> s);
+            const uint64_t pg = ((x << s) + (r & ((1u << s) - 1))) << o;
+            st_rlx32(&h->kind[pg], kKindTree | (uint32_t)o);
+            my = pg << kPageShift;
+        }
+        served += cap < N - served ? cap : N - served;
+    }
+    return my;
+}
+
+// ---- the entry points ---------------------------------------------------------
+static __device__ __noinline__ uint64_t ga_malloc_off(const ga_desc* h, uint64_t n) {
+    const unsigned act = __activemask();
+    const int key = size_key(h, n);
+    const unsigned grp = __match_any_sync(act, key);
+    if (key < 0) return kNull;
+    uint64_t my;
+    if (key < kNcls) {
+        const uint32_t A = arena_of(h);
+        const uint32_t N = __popc(grp), slots = slots_of(key);
+        const int leader = __ffs(grp) - 1;
+        int r = 0;
+        if ((int)lane_id() == leader)
+            r = bsem_wait(sem_ptr(h, A, key), N, slots * ((N + slots - 1) / slots), ArenaSpin{h, A});
+        r = __shfl_sync(grp, r, leader);
+        my = r == kAcquired ? bin_claim_collective(h, grp, A, key) : bin_grow_collective(h, grp, A, key);
+        if (__any_sync(grp, my == kNull)) {                 // R-27: degrade to per-lane waits
+            if ((int)lane_id() == leader) stat_add(h, kStatFallback, 1);
+            if (my == kNull) my = bin_malloc_lane(h, A, key);
+        }
+    } else {
+        const int o = key - kNcls;
+        my = tree_malloc_group(h, grp, o);
+        if (my == kNull) {
+            int64_t x = tree_alloc_one_retry(h, o);
+            if (x >= 0) {
+                uint64_t pg = (uint64_t)x << o;
                 st_rlx32(&h->kind[pg], kKindTree | (uint32_t)o);
                 my = pg << kPageShift;
-            }
+            } else stat_add(h, kStatFail, 1);
         }
     }
     return my;
 }
 
-static __device__ __noinline__ uint64_t ga_malloc_off(const ga_desc* h, uint64_t n) {
-    unsigned act = __activemask();
-    int key = size_key(h, n);
-    unsigned grp = __match_any_sync(act, key);
-    if (key < 0) return kNull;
-    return group_malloc(h, grp, key);
-}
-
-// free: TBuddy blocks per lane; bin slots grouped per bitmap word (one
-// atomicAnd) and per (arena, class) (one signal)
+// free: TBuddy blocks merge inside the warp first (lanes freeing sibling blocks
+// pair up with __match_any_sync and continue with the parent -- a collective
+// free), then each surviving block runs the merge-on-free protocol; bin slots
+// are grouped per bitmap word (one atomicAnd) and per (arena, class) (one signal).
 static __device__ __noinline__ void ga_free_off(const ga_desc* h, uint64_t off) {
-    unsigned act = __activemask();
+    const unsigned act = __activemask();
     uint32_t k = 0;
     uint64_t p = 0;
     if (off != kNull) { p = off >> kPageShift; k = ld_rlx32(&h->kind[p]); }
-    bool is_bin = (off != kNull) && ((k & 0xC0000000u) == kKindBin);
-    unsigned bins = __ballot_sync(act, is_bin);
-    if (off != kNull && !is_bin) {
-        // TBuddy block (page aligned); order from the page kind (R-18)
-        int o = (int)(k & 0xFF);
+    const bool is_bin = (off != kNull) && ((k & 0xC0000000u) == kKindBin);
+    const bool is_tree = (off != kNull) && !is_bin;
+    const unsigned bins = __ballot_sync(act, is_bin);
+    const unsigned trees = __ballot_sync(act, is_tree);
+    if (is_tree) {
+        int n = (int)(k & 0xFF);                               // order from the page kind (R-18)
+        uint64_t x = p >> n;
         st_rlx32(&h->kind[p], 0);
         fence();
-        tree_free(h, o, p >> o);
+        unsigned part = trees;
+        bool alive = true;
+        for (;;) {
+            const uint64_t key = ((uint64_t)n << 58) | (x >> 1);
+            const unsigned mm = __match_any_sync(part, key);
+            const bool paired = __popc(mm) == 2;
+            if (!__any_sync(part, paired)) break;
+            if (paired) {
+                if ((int)lane_id() == __ffs(mm) - 1) { x >>= 1; n++; }   // both halves are ours: merged
+                else alive = false;
+            }
+            part = __ballot_sync(part, alive);
+            if (!alive) break;
+        }
+        if (alive) tree_free(h, n, x);
+        return;
     }
     if (!is_bin) return;
-    uint32_t A = (k >> 8) & 0xFFFFu;
-    int c = (int)(k & 0xFF);
-    uint32_t slot = (uint32_t)((off & (kPage - 1)) >> (c + kMinShift));
-    int w = (int)(slot >> 6);
-    uint64_t key1 = (p << 2) | (uint64_t)w;
-    unsigned g1 = __match_any_sync(bins, key1);
-    uint64_t bit = 1ull << (slot & 63);
-    uint32_t lo = __reduce_or_sync(g1, (uint32_t)bit), hi = __reduce_or_sync(g1, (uint32_t)(bit >> 32));
-    uint64_t mask = ((uint64_t)hi << 32) | lo;
+    const uint32_t A = (k >> 8) & 0xFFFFu;
+    const int c = (int)(k & 0xFF);
+    const uint32_t slot = (uint32_t)((off & (kPage - 1)) >> (c + kMinShift));
+    const int w = (int)(slot >> 6);
+    const unsigned g1 = __match_any_sync(bins, (p << 2) | (uint64_t)w);
+    const uint64_t bit = 1ull << (slot & 63);
+    const uint64_t mask = ((uint64_t)__reduce_or_sync(g1, (uint32_t)(bit >> 32)) << 32) | __reduce_or_sync(g1, (uint32_t)bit);
     if ((int)lane_id() == __ffs(g1) - 1) {
         uint64_t* bw = page_bits(h, p);
-        uint64_t old = a_and(&bw[w], ~mask);
-        uint64_t v = valid_mask(c, w);
-        if ((old | ~v) == ~0ull) nonfull_set(h, p, c);    // the word was full: bin back in the list
-        if (((old & ~mask) & v) == 0) {                    // this word is empty: is the bin?
+        const uint64_t old = a_and(&bw[w], ~mask);
+        const uint64_t v = valid_mask(c, w);
+        if ((old | ~v) == ~0ull) nonfull_set(h, p, c, A);     // the word was full: bin back in the list
+        if (((old & ~mask) & v) == 0) {                        // this word is empty: is the bin?
             uint64_t ww[4];
             ld_bitmap(bw, ww);
             bool empty = true;
@@ -1088,8 +1034,7 @@ static __device__ __noinline__ void ga_free_off(const ga_desc* h, uint64_t off) 
         }
     }
     __syncwarp(bins);
-    uint32_t key2 = (A << 3) | (uint32_t)c;
-    unsigned g2 = __match_any_sync(bins, key2);
+    const unsigned g2 = __match_any_sync(bins, (A << 3) | (uint32_t)c);
     if ((int)lane_id() == __ffs(g2) - 1) bsem_signal_after_rmw(sem_ptr(h, A, c), __popc(g2));
 }
 

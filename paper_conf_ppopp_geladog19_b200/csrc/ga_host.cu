@@ -50,10 +50,11 @@ __global__ void k_quiesce_chunks(const ga_desc* h) {
         if (h->chunk_owner[ch] != 0 && ld_rlx(&h->chunk_used[ch]) == 0) chunk_release(h, ch);
     }
 }
+// quiesce step 3: no candidate can remain (every empty bin was reclaimed)
 __global__ void k_quiesce_clear(const ga_desc* h) {
     uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     if (i < h->nchunks) h->chunk_cand[i] = 0;
-    if (i < h->n_arenas) h->cand_any[i * kSemStride] = 0;
+    if (i < (uint64_t)h->n_arenas * h->ahb_words) h->ahb[(i / h->ahb_words) * kAhbPerArena * h->ahb_words + kAhbCnd * h->ahb_words + i % h->ahb_words] = 0;
 }
 
 inline int grid_for(uint64_t n) { uint64_t b = (n + 255) / 256; return (int)(b > 4096 ? 4096 : (b ? b : 1)); }
@@ -70,8 +71,7 @@ ga_status init_heap(ga_heap_t h, cudaStream_t s) {
     k_fill_u64<<<grid_for((uint64_t)d.n_arenas * kNcls * kSemStride), 256, 0, s>>>(d.sem, (uint64_t)d.n_arenas * kNcls * kSemStride, sem_word(0, 0));
     k_fill_u64<<<grid_for((uint64_t)d.n_arenas * kSemStride), 256, 0, s>>>(d.psem, (uint64_t)d.n_arenas * kSemStride, sem_word(0, 0));
     k_fill_u32<<<grid_for((uint64_t)d.n_arenas * kNcls), 256, 0, s>>>(d.hint, (uint64_t)d.n_arenas * kNcls, 0xFFFFFFFFu);
-    k_fill_u64<<<grid_for(h->owned_words), 256, 0, s>>>(d.owned, h->owned_words, 0ull);
-    k_fill_u64<<<grid_for((uint64_t)d.n_arenas * kSemStride), 256, 0, s>>>(d.cand_any, (uint64_t)d.n_arenas * kSemStride, 0ull);
+    k_fill_u64<<<grid_for(h->ahb_total_words), 256, 0, s>>>(d.ahb, h->ahb_total_words, 0ull);
     k_fill_u64<<<1, 32, 0, s>>>(d.stats, 16, 0ull);
     if (!chk(cudaGetLastError())) return GA_ECUDA;
     if (!chk(cudaMemcpyAsync(h->ddesc, &h->dev, sizeof(ga_desc), cudaMemcpyHostToDevice, s))) return GA_ECUDA;
@@ -81,13 +81,13 @@ ga_status init_heap(ga_heap_t h, cudaStream_t s) {
     return GA_OK;
 }
 
+// set bit i of a 3-level bitset image [w0 | w1 | w2] (section 3 of ga_device_impl.cuh)
 void hb_host_set(std::vector<uint64_t>& img, uint64_t base, uint32_t n0, uint64_t i) {
-    HB b = hb_make(nullptr, n0);
-    uint64_t j = i;
-    for (int k = 0; k < b.nl; k++) {
-        img[base + b.off[k] + (j >> 6)] |= 1ull << (j & 63);
-        j >>= 6;
-    }
+    img[base + (i >> 6)] |= 1ull << (i & 63);
+    uint64_t j = i >> 6;
+    img[base + n0 + (j >> 6)] |= 1ull << (j & 63);
+    uint64_t j1 = j >> 6;
+    img[base + n0 + hb3_n1(n0) + (j1 >> 6)] |= 1ull << (j1 & 63);
 }
 
 }  // namespace
@@ -147,10 +147,11 @@ ga_status ga_heap_create(int device, ga_stream_t stream, void* buf, size_t bytes
         uint64_t bits = 1ull << (L - n);
         d.lvl_words[n] = (uint32_t)((bits + 63) / 64);
         d.lvl_off[n] = aw;
-        aw += hb_total_words(d.lvl_words[n]);
+        aw += hb3_words(d.lvl_words[n]);
     }
     h->avail_words = aw;
-    h->owned_words = (uint64_t)d.n_arenas * hb_total_words(d.chunk_words);
+    d.ahb_words = hb3_words(d.chunk_words);
+    h->ahb_total_words = (uint64_t)d.n_arenas * kAhbPerArena * d.ahb_words;
     Carve cv;
     uint64_t o_desc = cv.take<ga_desc>(1);
     uint64_t o_bits = cv.take<uint64_t>(d.pages * kBinWords);
@@ -162,8 +163,7 @@ ga_status ga_heap_create(int device, ga_stream_t stream, void* buf, size_t bytes
     uint64_t o_sem = cv.take<uint64_t>((uint64_t)d.n_arenas * kNcls * kSemStride);
     uint64_t o_psem = cv.take<uint64_t>((uint64_t)d.n_arenas * kSemStride);
     uint64_t o_hint = cv.take<uint32_t>((uint64_t)d.n_arenas * kNcls);
-    uint64_t o_owned = cv.take<uint64_t>(h->owned_words);
-    uint64_t o_any = cv.take<uint64_t>((uint64_t)d.n_arenas * kSemStride);
+    uint64_t o_owned = cv.take<uint64_t>(h->ahb_total_words);
     uint64_t o_avail = cv.take<uint64_t>(aw);
     uint64_t o_tsem = cv.take<uint64_t>((uint64_t)(L + 1) * kSemStride);
     uint64_t o_stats = cv.take<uint64_t>(16);
@@ -187,8 +187,7 @@ ga_status ga_heap_create(int device, ga_stream_t stream, void* buf, size_t bytes
     d.sem = (uint64_t*)(m + o_sem);
     d.psem = (uint64_t*)(m + o_psem);
     d.hint = (uint32_t*)(m + o_hint);
-    d.owned = (uint64_t*)(m + o_owned);
-    d.cand_any = (uint64_t*)(m + o_any);
+    d.ahb = (uint64_t*)(m + o_owned);
     d.avail = (uint64_t*)(m + o_avail);
     d.tsem = (uint64_t*)(m + o_tsem);
     d.stats = (uint64_t*)(m + o_stats);
@@ -251,7 +250,7 @@ ga_status ga_heap_quiesce(ga_heap_t h, ga_stream_t stream) {
     cudaStream_t s = (cudaStream_t)stream;
     k_quiesce_bins<<<grid_for(h->dev.pages), 256, 0, s>>>(h->ddesc);
     k_quiesce_chunks<<<grid_for(h->dev.nchunks), 256, 0, s>>>(h->ddesc);
-    uint64_t n = h->dev.nchunks > h->dev.n_arenas ? h->dev.nchunks : h->dev.n_arenas;
+    uint64_t n = h->dev.nchunks > (uint64_t)h->dev.n_arenas * h->dev.ahb_words ? h->dev.nchunks : (uint64_t)h->dev.n_arenas * h->dev.ahb_words;
     k_quiesce_clear<<<(int)((n + 255) / 256), 256, 0, s>>>(h->ddesc);
     return cudaGetLastError() == cudaSuccess ? GA_OK : GA_ECUDA;
 }

@@ -16,7 +16,7 @@ struct ga_heap_s {
     std::vector<uint64_t> avail_init;   // host image of the tree bitmaps (empty heap)
     std::vector<uint64_t> tsem_init;
     uint64_t avail_words = 0;
-    uint64_t owned_words = 0;
+    uint64_t ahb_total_words = 0;
     uint64_t peak_reserved_pages = 0;
     void* scratch = nullptr;       // device scratch for ga_trace_timed_host
     size_t scratch_bytes = 0;
