@@ -792,8 +792,8 @@ static __device__ __noinline__ uint64_t bin_claim_collective(const ga_desc* h, u
     const uint32_t per_page = slots_of(c) < 64 ? slots_of(c) : 64;
     const uint64_t csz = 16ull << c;
     uint64_t my = kNull;
-    unsigned unsat = grp;
-    while (unsat) {
+    unsigned unsat = grp;                                   // lanes still without a slot (this lane included)
+    for (;;) {
         const int L = __ffs(unsat) - 1;
         uint64_t ch = 0, m = 0;
         if ((int)lane == L) ch = bin_find_chunk(h, A, c, &m);
@@ -812,6 +812,7 @@ static __device__ __noinline__ uint64_t bin_claim_collective(const ga_desc* h, u
         const uint32_t pr = __popc(pg & lanemask_lt());
         if (pr < (uint32_t)__popcll(got)) my = (page << kPageShift) + (uint64_t)(wi * 64 + nth_set(got, pr)) * csz;
         unsat = __ballot_sync(unsat, my == kNull);
+        if (my != kNull) break;                             // a satisfied lane leaves the group
     }
     return my;
 }
