@@ -50,6 +50,7 @@ constexpr uint32_t kKindBin = 0x40000000u;      // | arena << 8 | class
 constexpr uint32_t kKindTree = 0x80000000u;     // | order
 constexpr int kSemStride = 4;                   // u64 words between semaphores (32 B)
 constexpr int kMaxLevels = 48;
+constexpr uint32_t kReclaimKeep = 64;           // free slots a delegated reclaim leaves per class
 
 enum { kStatBinGrow = 0, kStatChunkGrow, kStatBinReclaim, kStatChunkReclaim, kStatFallback,
        kStatFail, kNumStats };
@@ -143,11 +144,12 @@ static __device__ __forceinline__ void bsem_signal_after_rmw(uint64_t* s, uint32
 
 // try-wait (R-7): C -= N iff C >= N.  One fetch-add: subtract,
 // and give the units back if the pre-image was short.
-static __device__ __forceinline__ bool bsem_trywait(uint64_t* s, uint32_t N) {
-    if (sem_C(ld_rlx(s)) < (int32_t)N) return false;
+static __device__ __forceinline__ bool bsem_trywait(uint64_t* s, uint32_t N, uint32_t keep = 0) {
+    // keep: succeed only if at least `keep` further units stay behind
+    if (sem_C(ld_rlx(s)) < (int32_t)(N + keep)) return false;
     const uint64_t dn = (uint64_t)N << 32;
     uint64_t old = a_add(s, (uint64_t)0 - dn);
-    if (sem_C(old) >= (int32_t)N) return true;
+    if (sem_C(old) >= (int32_t)(N + keep)) return true;
     a_add(s, dn);
     return false;
 }
@@ -427,11 +429,11 @@ static __device__ __forceinline__ bool page_full(const uint64_t w[4], int c) {
     return true;
 }
 
-static __device__ void reclaim_arena(const ga_desc* h, uint32_t A, int budget);
+static __device__ void reclaim_arena(const ga_desc* h, uint32_t A, int budget, uint32_t keep);
 // delegated work run by threads blocked in an arena semaphore wait (Sec. 4.2.1)
 struct ArenaSpin {
     const ga_desc* h; uint32_t A;
-    __device__ void operator()() const { reclaim_arena(h, A, 4); }
+    __device__ void operator()() const { reclaim_arena(h, A, 4, kReclaimKeep); }
 };
 
 // page p (class c, arena A) has a free slot again
@@ -458,8 +460,9 @@ static __device__ __noinline__ void nonfull_clear_if_full(const ga_desc* h, uint
 }
 
 // Take a new chunk from TBuddy for arena A, keep its first k pages, open the rest.
+static __device__ __noinline__ int64_t tree_alloc_one_retry(const ga_desc* h, int o);
 static __device__ __noinline__ int64_t chunk_acquire(const ga_desc* h, uint32_t A, uint32_t k) {
-    int64_t ch = tree_alloc_one(h, kChunkOrder);
+    int64_t ch = tree_alloc_one_retry(h, kChunkOrder);
     if (ch < 0) return -1;
     st_rlx32(&h->chunk_owner[ch], A + 1);
     fence();
@@ -623,8 +626,10 @@ static __device__ __noinline__ uint64_t bin_find_chunk(const ga_desc* h, uint32_
 // failing mallocs and ga_heap_quiesce do the reclaiming.
 // ---------------------------------------------------------------------------
 // Reclaim page p if it is an empty bin: try-wait all its slots (R-22), then take
-// every slot word with a CAS (all free -> all ones).
-static __device__ __noinline__ bool bin_reclaim(const ga_desc* h, uint64_t p) {
+// every slot word with a CAS (all free -> all ones).  `keep`: leave at least
+// that many free slots of the class behind -- delegated reclamation must not
+// take the bins the waiting threads are about to use (0 for quiesce).
+static __device__ __noinline__ bool bin_reclaim(const ga_desc* h, uint64_t p, uint32_t keep) {
     uint32_t k = ld_rlx32(&h->kind[p]);
     if ((k & 0xC0000000u) != kKindBin) return false;
     uint32_t A = (k >> 8) & 0xFFFFu;
@@ -634,7 +639,7 @@ static __device__ __noinline__ bool bin_reclaim(const ga_desc* h, uint64_t p) {
     ld_bitmap(bw, w);
     for (int i = 0; i < words_of(c); i++) if (w[i] & valid_mask(c, i)) return false;
     uint32_t slots = slots_of(c);
-    if (!bsem_trywait(sem_ptr(h, A, c), slots)) return false;
+    if (!bsem_trywait(sem_ptr(h, A, c), slots, keep)) return false;
     int i = 0;
     for (; i < words_of(c); i++) {
         uint64_t v = valid_mask(c, i);
@@ -663,8 +668,9 @@ static __device__ __forceinline__ void mark_candidate(const ga_desc* h, uint64_t
     if (a_or(cw, bit) == 0) hb3_set(arena_hb(h, A, kAhbCnd), p >> kChunkShift);
 }
 
-// Reclaim up to `budget` candidate bins of arena A (budget < 0: all).
-static __device__ __noinline__ void reclaim_arena(const ga_desc* h, uint32_t A, int budget) {
+// Reclaim up to `budget` candidate bins of arena A (budget < 0: all), leaving
+// at least `keep` free slots per class (0: reclaim every empty bin).
+static __device__ __noinline__ void reclaim_arena(const ga_desc* h, uint32_t A, int budget, uint32_t keep) {
     HB3 cb = arena_hb(h, A, kAhbCnd);
     if (!hb3_any(cb)) return;
     uint32_t seed = scatter_seed();
@@ -676,17 +682,32 @@ static __device__ __noinline__ void reclaim_arena(const ga_desc* h, uint32_t A, 
         uint64_t ch = (uint64_t)j * 64 + (uint64_t)(__ffsll((long long)cm) - 1);
         uint64_t pm = a_exch(&h->chunk_cand[ch], 0);
         hb3_clear_summarised(cb, ch, &h->chunk_cand[ch], 0);
+        uint64_t pm_left = 0;
         while (pm) {
             uint32_t pb = (uint32_t)(__ffsll((long long)pm) - 1);
             pm &= pm - 1;
             if (budget == 0) { mark_candidate(h, ch * kChunkPages + pb, A); continue; }
-            bin_reclaim(h, ch * kChunkPages + pb);
+            if (!bin_reclaim(h, ch * kChunkPages + pb, keep)) {
+                // still empty but the class needs it for now: keep it a candidate
+                uint64_t w[4];
+                ld_bitmap(page_bits(h, ch * kChunkPages + pb), w);
+                if (ld_rlx32(&h->kind[ch * kChunkPages + pb]) & kKindBin) {
+                    int c = (int)(ld_rlx32(&h->kind[ch * kChunkPages + pb]) & 0xFF);
+                    bool empty = true;
+                    for (int i = 0; i < words_of(c); i++) if (w[i] & valid_mask(c, i)) empty = false;
+                    if (empty) { pm_left |= 1ull << pb; }
+                }
+            }
             if (budget > 0) budget--;
+        }
+        if (pm_left) {                                      // re-mark what could not go yet
+            if (a_or(&h->chunk_cand[ch], pm_left) == 0) hb3_set(cb, ch);
+            return;                                         // and stop: the rest is in use too
         }
     }
 }
 static __device__ __noinline__ void reclaim_all(const ga_desc* h) {
-    for (uint32_t A = 0; A < h->n_arenas; A++) reclaim_arena(h, A, -1);
+    for (uint32_t A = 0; A < h->n_arenas; A++) reclaim_arena(h, A, -1, 0);
 }
 
 // Per-lane TBuddy allocation with the no-false-starvation retry: the optimistic
@@ -748,7 +769,7 @@ static __device__ __noinline__ uint64_t bin_malloc_lane(const ga_desc* h, uint32
             uint64_t pm = page_claim(h, A0, 1, &ch);
             p = ch * kChunkPages + (uint64_t)(__ffsll((long long)pm) - 1);
         } else {
-            reclaim_arena(h, A0, -1);
+            reclaim_arena(h, A0, -1, kReclaimKeep);
             int64_t ch = chunk_acquire(h, A0, 1);
             if (ch >= 0) { bsem_signal(psem_ptr(h, A0), kChunkPages - 1, kChunkPages - 1); p = (uint64_t)ch * kChunkPages; }
             else bsem_signal(psem_ptr(h, A0), 0, kChunkPages - 1);
@@ -837,7 +858,7 @@ static __device__ __noinline__ uint64_t bin_grow_collective(const ga_desc* h, un
     uint64_t ch = 0, pm = 0;
     if ((int)lane == leader) {
         if (bsem_wait(psem_ptr(h, A), k, kChunkPages, ArenaSpin{h, A}) == kGrow) {
-            reclaim_arena(h, A, -1);                                         // delegated work first
+            reclaim_arena(h, A, -1, kReclaimKeep);                           // delegated work first
             int64_t nc = chunk_acquire(h, A, k);
             if (nc < 0) {
                 bsem_signal(psem_ptr(h, A), 0, kChunkPages - k);
@@ -895,20 +916,29 @@ static __device__ __noinline__ uint64_t tree_malloc_group(const ga_desc* h, unsi
     int m = o;
     uint32_t Nm = N;
     if ((int)lane == leader) {
-        for (;;) {
-            if (m > (int)h->L) {
-                uint32_t nk = N;
-                for (int k = o; k < m; k++) { bsem_signal(tsem_ptr(h, k), 0, 2 * ((nk + 1) >> 1) - nk); nk = (nk + 1) >> 1; }
-                m = -1;
-                break;
+        uint32_t ns = 128;
+        for (int attempt = 0;; attempt++) {
+            m = o; Nm = N;
+            for (;;) {
+                if (m > (int)h->L) {                         // nothing to grow from: retract every E
+                    uint32_t nk = N;
+                    for (int k = o; k < m; k++) { bsem_signal(tsem_ptr(h, k), 0, 2 * ((nk + 1) >> 1) - nk); nk = (nk + 1) >> 1; }
+                    m = -1;
+                    break;
+                }
+                if (bsem_wait_fast(tsem_ptr(h, m), Nm, 2 * ((Nm + 1) >> 1), NoSpin()) == kAcquired) break;
+                Nm = (Nm + 1) >> 1;
+                m++;
             }
-            if (bsem_wait_fast(tsem_ptr(h, m), Nm, 2 * ((Nm + 1) >> 1), NoSpin()) == kAcquired) break;
-            Nm = (Nm + 1) >> 1;
-            m++;
+            // No false resource starvation: while splits are in flight
+            // below the top (C >= 1 or D != 0 at some order >= o), wait and re-climb
+            if (m >= 0 || attempt >= 4096 || !tree_has_supply(h, o)) break;
+            __nanosleep(ns); if (ns < 8192) ns <<= 1;
         }
     }
     m = __shfl_sync(grp, m, leader);
     if (m < 0) return kNull;
+    Nm = __shfl_sync(grp, Nm, leader);
     const int s = m - o;
     uint64_t my = kNull;
     uint32_t served = 0;

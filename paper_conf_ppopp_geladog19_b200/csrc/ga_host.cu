@@ -41,7 +41,7 @@ __global__ void k_fill_u32(uint32_t* p, uint64_t n, uint32_t v) {
 __global__ void k_quiesce_bins(const ga_desc* h) {
     for (uint64_t p = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; p < h->pages; p += (uint64_t)gridDim.x * blockDim.x) {
         uint32_t k = h->kind[p];
-        if ((k & 0xC0000000u) == kKindBin) bin_reclaim(h, p);
+        if ((k & 0xC0000000u) == kKindBin) bin_reclaim(h, p, 0);
     }
 }
 // quiesce step 2: chunks whose pages are all free go back to TBuddy
