@@ -150,6 +150,42 @@ def config_of(trace, args):
             "block": args.block, "l2": "flushed between steps (512 MiB write)", "seed": hex(trace.seed)}
 
 
+def d3_sweep(ga, heap, stream, dev, T, args, sizes=(16, 32, 64, 128, 256, 512, 1024, 2048, 4096, 8192), R=16):
+    import torch
+    res = {}
+    cc = torch.zeros(8, dtype=torch.int64, device=dev)
+    for sz in sizes:
+        d = torch.full((R * T,), sz, dtype=torch.int32, device=dev)
+        heap.reset()
+        times = []
+        for rep in range(4):
+            cc.zero_()
+            a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a0.record(stream)
+            ga.ga_trace_timed(heap.h, stream.cuda_stream, d.data_ptr(), R, T, 0, cc.data_ptr(), args.block)
+            a1.record(stream)
+            a1.synchronize()
+            if rep:
+                times.append(a0.elapsed_time(a1) / 1e3)
+        c = cc.cpu().numpy()
+        ours = float(c[0] + c[2]) / (sum(times) / len(times))
+        fails = int(c[1])
+        cc.zero_()
+        a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a0.record(stream)
+        ga.ga_cuda_trace_timed(stream.cuda_stream, d.data_ptr(), 1, T, 0, cc.data_ptr(), args.block)
+        a1.record(stream)
+        a1.synchronize()
+        c = cc.cpu().numpy()
+        cuda = float(c[0] + c[2]) / (a0.elapsed_time(a1) / 1e3)
+        res[str(sz)] = {"ours": ours, "cuda_malloc": cuda, "speedup": ours / cuda, "ours_failed": fails,
+                        "cuda_failed": int(c[1]), "ours_rounds": R, "cuda_rounds": 1}
+    vals = [v["speedup"] for v in res.values()]
+    res["min_speedup"] = min(vals)
+    res["geomean_speedup"] = float(np.exp(np.mean(np.log(vals))))
+    return res
+
+
 # ----------------------------------------------------------------------------- our arm
 def main():
     ap = argparse.ArgumentParser()
@@ -338,6 +374,10 @@ def main():
                               "failed_mallocs": int(ccn[1]), "seconds": t_cuda,
                               "heap_limit_bytes": trace.heap_bytes}
         out["speedup_vs_cuda_malloc"] = value / cuda_rate
+
+        # ---- d3: warp-uniform sizes 16 B - 8 KiB (BASELINE configs[2]), malloc+free per
+        # thread and round (D = 0), full grid; CUDA malloc on a bounded prefix of rounds
+        out["d3_sweep"] = d3_sweep(ga, heap, stream, dev, T, args)
 
     print(json.dumps(out), flush=True)
     if dist:

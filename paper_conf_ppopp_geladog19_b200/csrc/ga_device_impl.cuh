@@ -409,12 +409,13 @@ static __device__ __noinline__ void tree_free(const ga_desc* h, int n, uint64_t 
     }
 }
 
-// Does any order >= o show a unit (C >= 1) or growth / reservations in flight
-// (D != 0)?  At true exhaustion every such word is (0, 0).
+// Does any order >= o show a unit (C >= 1) or expected units nobody has
+// reserved yet (D = E - R > 0, a split in flight)?  The caller has retracted
+// its own E first.  At true exhaustion every such word shows C = 0, D <= 0.
 static __device__ __noinline__ bool tree_has_supply(const ga_desc* h, int o) {
     for (int k = o; k <= (int)h->L; k++) {
         uint64_t w = ld_rlx(tsem_ptr(h, k));
-        if (sem_C(w) >= 1 || sem_D(w) != 0) return true;
+        if (sem_C(w) >= 1 || sem_D(w) > 0) return true;
     }
     return false;
 }
@@ -716,7 +717,7 @@ static __device__ __noinline__ void reclaim_all(const ga_desc* h) {
 static __device__ __noinline__ int64_t tree_alloc_one_retry(const ga_desc* h, int o) {
     bool drained = false;
     uint32_t ns = 64;
-    for (int attempt = 0; attempt < 256; attempt++) {
+    for (int attempt = 0; attempt < 64; attempt++) {
         int64_t x = tree_alloc_one(h, o);
         if (x >= 0) return x;
         if (!tree_has_supply(h, o)) {
@@ -932,7 +933,7 @@ static __device__ __noinline__ uint64_t tree_malloc_group(const ga_desc* h, unsi
             }
             // No false resource starvation: while splits are in flight
             // below the top (C >= 1 or D != 0 at some order >= o), wait and re-climb
-            if (m >= 0 || attempt >= 4096 || !tree_has_supply(h, o)) break;
+            if (m >= 0 || attempt >= 64 || !tree_has_supply(h, o)) break;
             __nanosleep(ns); if (ns < 8192) ns <<= 1;
         }
     }
