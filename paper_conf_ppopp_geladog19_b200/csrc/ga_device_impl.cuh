@@ -409,13 +409,15 @@ static __device__ __noinline__ void tree_free(const ga_desc* h, int n, uint64_t 
     }
 }
 
-// Does any order >= o show a unit (C >= 1) or expected units nobody has
-// reserved yet (D = E - R > 0, a split in flight)?  The caller has retracted
-// its own E first.  At true exhaustion every such word shows C = 0, D <= 0.
-static __device__ __noinline__ bool tree_has_supply(const ga_desc* h, int o) {
+// Supply visible to a failed climber (after it retracted its own E):
+//   units  -- some order k >= o holds an available node now (C >= 1);
+//   growth -- some order k >= o expects units nobody reserved yet (D > 0).
+// At true exhaustion both are false.  Growth also counts other failing
+// climbers' transient E, so only the first retries may wait on it.
+static __device__ __noinline__ bool tree_has_supply(const ga_desc* h, int o, bool count_growth) {
     for (int k = o; k <= (int)h->L; k++) {
         uint64_t w = ld_rlx(tsem_ptr(h, k));
-        if (sem_C(w) >= 1 || sem_D(w) > 0) return true;
+        if (sem_C(w) >= 1 || (count_growth && sem_D(w) > 0)) return true;
     }
     return false;
 }
@@ -717,12 +719,12 @@ static __device__ __noinline__ void reclaim_all(const ga_desc* h) {
 static __device__ __noinline__ int64_t tree_alloc_one_retry(const ga_desc* h, int o) {
     bool drained = false;
     uint32_t ns = 64;
-    for (int attempt = 0; attempt < 64; attempt++) {
+    for (int attempt = 0; attempt < 32; attempt++) {
         int64_t x = tree_alloc_one(h, o);
         if (x >= 0) return x;
-        if (!tree_has_supply(h, o)) {
+        if (!tree_has_supply(h, o, attempt < 2)) {
             if (drained) return -1;
-            reclaim_all(h);
+            reclaim_all(h);                                     // empty bins / chunks back to the tree
             drained = true;
             continue;
         }
@@ -787,6 +789,8 @@ static __device__ __noinline__ uint64_t bin_malloc_lane(const ga_desc* h, uint32
     }
     for (uint32_t t = 1; t <= h->n_arenas; t++) {
         uint32_t B = (A0 + t) % h->n_arenas;
+        uint64_t pw = ld_rlx(psem_ptr(h, B));
+        if (sem_C(pw) < 1 && (int64_t)sem_C(pw) + sem_D(pw) < 1) continue;    // nothing there or expected
         if (bsem_wait(psem_ptr(h, B), 1, 1, NoSpin()) == kAcquired) {
             uint64_t ch;
             uint64_t pm = page_claim(h, B, 1, &ch);
@@ -799,6 +803,8 @@ static __device__ __noinline__ uint64_t bin_malloc_lane(const ga_desc* h, uint32
     }
     for (uint32_t t = 1; t <= h->n_arenas; t++) {
         uint32_t B = (A0 + t) % h->n_arenas;
+        uint64_t cw = ld_rlx(sem_ptr(h, B, c));
+        if (sem_C(cw) < 1 && (int64_t)sem_C(cw) + sem_D(cw) < 1) continue;
         if (bsem_wait(sem_ptr(h, B, c), 1, 1, NoSpin()) == kAcquired) return bin_claim_one(h, B, c);
     }
     stat_add(h, kStatFail, 1);
@@ -932,8 +938,8 @@ static __device__ __noinline__ uint64_t tree_malloc_group(const ga_desc* h, unsi
                 m++;
             }
             // No false resource starvation: while splits are in flight
-            // below the top (C >= 1 or D != 0 at some order >= o), wait and re-climb
-            if (m >= 0 || attempt >= 64 || !tree_has_supply(h, o)) break;
+            // (cold start) or units are visible at some order >= o, re-climb
+            if (m >= 0 || attempt >= 8 || !tree_has_supply(h, o, attempt < 2)) break;
             __nanosleep(ns); if (ns < 8192) ns <<= 1;
         }
     }

@@ -16,9 +16,13 @@ ap.add_argument("--size", type=int, default=16)
 ap.add_argument("--rounds", type=int, default=16)
 ap.add_argument("--reps", type=int, default=3)
 ap.add_argument("--cuda", action="store_true")
+ap.add_argument("--kmin", type=int, default=3)
+ap.add_argument("--kmax", type=int, default=15)
 a = ap.parse_args()
 if a.workload == "d4":
     t = tracegen.d4_mixed("pressure", R=a.rounds)
+    if (a.kmin, a.kmax) != (3, 15):
+        t = tracegen.Trace("d4_sub", tracegen.mixed_sizes(t.seed, a.rounds, t.T, a.kmin, a.kmax), 1, t.heap_bytes, t.seed)
 else:
     t = tracegen.d3_uniform(a.size, R=a.rounds)
 torch.cuda.set_device(0)
