@@ -72,6 +72,7 @@ typedef struct ga_desc {
     uint32_t pad0;
     uint64_t lvl_off[48];     /* word offset of level n in avail                        */
     uint32_t lvl_words[48];   /* u64 words of level n's availability bits               */
+    uint32_t* lvl_hint;       /* [48] last level-n word a claim succeeded in            */
 } ga_desc;
 
 /* Plain-old-data handle passed BY VALUE to kernels that call ga_malloc /

@@ -144,6 +144,15 @@ static __device__ __forceinline__ void bsem_signal_after_rmw(uint64_t* s, uint32
 
 // try-wait (R-7): C -= N iff C >= N.  One fetch-add: subtract,
 // and give the units back if the pre-image was short.
+// one fetch-add, no pre-load (callers that expect success, e.g. a merge whose
+// buddy bit was just seen set)
+static __device__ __forceinline__ bool bsem_trywait_direct(uint64_t* s, uint32_t N) {
+    const uint64_t dn = (uint64_t)N << 32;
+    uint64_t old = a_add(s, (uint64_t)0 - dn);
+    if (sem_C(old) >= (int32_t)N) return true;
+    a_add(s, dn);
+    return false;
+}
 static __device__ __forceinline__ bool bsem_trywait(uint64_t* s, uint32_t N, uint32_t keep = 0) {
     // keep: succeed only if at least `keep` further units stay behind
     if (sem_C(ld_rlx(s)) < (int32_t)(N + keep)) return false;
@@ -205,11 +214,11 @@ static __device__ __noinline__ int bsem_wait_impl(uint64_t* s, uint32_t N, uint3
             return kGrow;
         }
         w = a_add(s, dn - (uint64_t)N) + dn - (uint64_t)N;                                     // C += N, R += N
-        uint32_t ns = 64;
+        uint32_t ns = 32;
         while (sem_C(w) < (int32_t)N && (int64_t)sem_C(w) + sem_D(w) >= 0) {                    // R-2
             spin();
             __nanosleep(ns);
-            if (ns < 2048) ns <<= 1;
+            if (ns < 256) ns <<= 1;                         // a split lands within a few round trips
             w = ld_rlx(s);
         }
         a_add(s, (uint64_t)N);                                                                  // R -= N
@@ -337,8 +346,10 @@ static __device__ __forceinline__ void tree_publish(const ga_desc* h, int n, uin
 static __device__ __noinline__ uint64_t tree_claim_word(const ga_desc* h, int n, int need, uint32_t seed, uint64_t* wj) {
     HB3 b = level_hb(h, n);
     uint32_t ns = 32;
+    int64_t j = ld_rlx32(&h->lvl_hint[n]);                   // the last word a claim succeeded in
+    if (j >= b.n0 || ld_rlx(&b.w0[j]) == 0) j = -1;
     for (;;) {
-        int64_t j = hb3_find(b, seed);
+        if (j < 0) j = hb3_find(b, seed);
         if (j >= 0) {
             uint64_t x = ld_rlx(&b.w0[j]);
             while (x) {
@@ -346,10 +357,15 @@ static __device__ __noinline__ uint64_t tree_claim_word(const ga_desc* h, int n,
                 uint64_t old = a_and(&b.w0[j], ~m);
                 uint64_t got = old & m;
                 if (old != 0 && (old & ~m) == 0) hb3_up_clear(b, (uint32_t)j);
-                if (got) { *wj = (uint64_t)j; return got; }
+                if (got) {
+                    if ((old & ~m) && ld_rlx32(&h->lvl_hint[n]) != (uint32_t)j) st_rlx32(&h->lvl_hint[n], (uint32_t)j);
+                    *wj = (uint64_t)j;
+                    return got;
+                }
                 x = old & ~m;
             }
         }
+        j = -1;
         __nanosleep(ns); if (ns < 1024) ns <<= 1;
         seed = hash32(seed + 1);
     }
@@ -388,7 +404,7 @@ static __device__ __noinline__ void tree_free(const ga_desc* h, int n, uint64_t 
         bool root = (n >= (int)h->L) || !node_inside(h, n, x ^ 1);
         uint64_t w = ld_rlx(wp);
         if (!root && (w & yb)) {
-            if (bsem_trywait(tsem_ptr(h, n), 1)) {
+            if (bsem_trywait_direct(tsem_ptr(h, n), 1)) {
                 uint64_t old = a_and(wp, ~yb);
                 if (old & yb) {                               // merged: free the parent at n + 1
                     if (old == yb) hb3_up_clear(b, (uint32_t)(x >> 6));
@@ -952,21 +968,24 @@ static __device__ __noinline__ uint64_t tree_malloc_group(const ga_desc* h, unsi
     uint32_t seed = scatter_seed();
     while (served < N) {
         uint64_t wj = 0, got = 0;
-        if ((int)lane == leader) {
-            uint32_t need_nodes = Nm - (served >> s);
-            got = tree_claim_word(h, m, (int)need_nodes, seed, &wj);
-            uint32_t nn = __popcll(got);
-            uint32_t rem = N - served;
-            if ((nn << s) >= rem && s > 0) {
-                // the last node is split: publish its unused right parts (E at each level)
-                uint64_t xlast = wj * 64 + (63 - __clzll((long long)got));
-                uint64_t pos = rem - ((nn - 1) << s);
-                for (int j = 0; j < s; j++)
-                    if ((pos >> j) & 1) { tree_publish(h, o + j, ((xlast << s) + pos) >> j, 1); pos += 1ull << j; }
-            }
-        }
+        if ((int)lane == leader) got = tree_claim_word(h, m, (int)(Nm - (served >> s)), seed, &wj);
         wj = __shfl_sync(grp, wj, leader);
         got = __shfl_sync(grp, got, leader);
+        {
+            const uint32_t nn = __popcll(got), rem = N - served;
+            if ((nn << s) >= rem && s > 0) {
+                // the last node is split: its unused right parts [pos, 2^s) decompose into
+                // one aligned block per set bit j of the running position (E at each level
+                // o + j); the group's lanes publish them in parallel, lane q doing level o + q
+                const uint64_t xlast = wj * 64 + (63 - __clzll((long long)got));
+                const uint64_t keep = rem - ((nn - 1) << s);
+                for (uint32_t j = rank; j < (uint32_t)s; j += N) {
+                    // running position before level j = keep rounded up to a multiple of 2^j
+                    const uint64_t pj = (keep + (1ull << j) - 1) & ~((1ull << j) - 1);
+                    if ((pj >> j) & 1) tree_publish(h, o + (int)j, ((xlast << s) + pj) >> j, 1);
+                }
+            }
+        }
         const uint32_t cap = (uint32_t)__popcll(got) << s;
         if (rank >= served && rank < served + cap) {
             const uint32_t r = rank - served;

@@ -73,6 +73,7 @@ ga_status init_heap(ga_heap_t h, cudaStream_t s) {
     k_fill_u32<<<grid_for((uint64_t)d.n_arenas * kNcls), 256, 0, s>>>(d.hint, (uint64_t)d.n_arenas * kNcls, 0xFFFFFFFFu);
     k_fill_u64<<<grid_for(h->ahb_total_words), 256, 0, s>>>(d.ahb, h->ahb_total_words, 0ull);
     k_fill_u64<<<1, 32, 0, s>>>(d.stats, 16, 0ull);
+    k_fill_u32<<<1, 64, 0, s>>>(d.lvl_hint, 48, 0u);
     if (!chk(cudaGetLastError())) return GA_ECUDA;
     if (!chk(cudaMemcpyAsync(h->ddesc, &h->dev, sizeof(ga_desc), cudaMemcpyHostToDevice, s))) return GA_ECUDA;
     if (!chk(cudaMemcpyAsync(d.avail, h->avail_init.data(), h->avail_words * 8, cudaMemcpyHostToDevice, s))) return GA_ECUDA;
@@ -167,6 +168,7 @@ ga_status ga_heap_create(int device, ga_stream_t stream, void* buf, size_t bytes
     uint64_t o_avail = cv.take<uint64_t>(aw);
     uint64_t o_tsem = cv.take<uint64_t>((uint64_t)(L + 1) * kSemStride);
     uint64_t o_stats = cv.take<uint64_t>(16);
+    uint64_t o_lhint = cv.take<uint32_t>(48);
     h->meta_bytes = cv.off;
     if (cudaMalloc(&h->meta, h->meta_bytes) != cudaSuccess) { delete h; cudaSetDevice(prev); return GA_ENOMEM; }
     if (buf) d.base = (char*)buf;
@@ -191,6 +193,7 @@ ga_status ga_heap_create(int device, ga_stream_t stream, void* buf, size_t bytes
     d.avail = (uint64_t*)(m + o_avail);
     d.tsem = (uint64_t*)(m + o_tsem);
     d.stats = (uint64_t*)(m + o_stats);
+    d.lvl_hint = (uint32_t*)(m + o_lhint);
     // empty heap: the binary decomposition of the pages into maximal aligned roots (R-30)
     h->avail_init.assign(aw, 0ull);
     h->tsem_init.assign((uint64_t)(L + 1) * kSemStride, 0ull);
