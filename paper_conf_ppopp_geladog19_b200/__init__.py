@@ -66,9 +66,11 @@ def lib():
     global _lib
     if _lib is not None:
         return _lib
-    path = _build.LIB
-    if not os.path.exists(path) or _build._stale():
-        path = _build.build()
+    path = os.environ.get("GA_LIB")            # a tuning variant built by _build.build(out=...)
+    if not path:
+        path = _build.LIB
+        if not os.path.exists(path) or _build._stale():
+            path = _build.build()
     L = ctypes.CDLL(path)
     vp, u32, u64, i32, sz = ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_int, ctypes.c_size_t
     P = ctypes.POINTER

@@ -50,6 +50,19 @@ constexpr uint32_t kKindBin = 0x40000000u;      // | arena << 8 | class
 constexpr uint32_t kKindTree = 0x80000000u;     // | order
 constexpr int kSemStride = 4;                   // u64 words between semaphores (32 B)
 constexpr int kMaxLevels = 48;
+// tuning switches; defaults are the measured best
+#ifndef GA_LVL_HINT
+#define GA_LVL_HINT 0            // 1: claim from the last successful level word first
+#endif
+#ifndef GA_TREE_SPIN_CAP
+#define GA_TREE_SPIN_CAP 256     // max __nanosleep backoff (ns) of a blocked TBuddy wait
+#endif
+#ifndef GA_OPT_LOAD_GATED
+#define GA_OPT_LOAD_GATED 0      // 1: optimistic (TBuddy) waits decide on a plain load first
+#endif
+#ifndef GA_MERGE_PRELOAD
+#define GA_MERGE_PRELOAD 1       // 1: try-wait loads the word before its fetch-add
+#endif
 constexpr uint32_t kReclaimKeep = 64;           // free slots a delegated reclaim leaves per class
 
 enum { kStatBinGrow = 0, kStatChunkGrow, kStatBinReclaim, kStatChunkReclaim, kStatFallback,
@@ -106,10 +119,17 @@ static __device__ __forceinline__ uint64_t lowest_bits(uint64_t x, int k) {
     return m;
 }
 // position of the n-th (0-based) set bit of x
+// (branch-free popc binary search; __fns is emulated with a loop on sm_100a)
 static __device__ __forceinline__ uint32_t nth_set(uint64_t x, uint32_t n) {
-    uint32_t lo = __popc((uint32_t)x);
-    if (n >= lo) { return 32 + __fns((uint32_t)(x >> 32), 0, (int)(n - lo) + 1); }
-    return __fns((uint32_t)x, 0, (int)n + 1);
+    uint32_t pos = 0, c;
+    c = __popc((uint32_t)x);          if (n >= c) { n -= c; x >>= 32; pos += 32; }
+    uint32_t v = (uint32_t)x;
+    c = __popc(v & 0xFFFFu);          if (n >= c) { n -= c; v >>= 16; pos += 16; }
+    c = __popc(v & 0xFFu);            if (n >= c) { n -= c; v >>= 8; pos += 8; }
+    c = __popc(v & 0xFu);             if (n >= c) { n -= c; v >>= 4; pos += 4; }
+    c = __popc(v & 0x3u);             if (n >= c) { n -= c; v >>= 2; pos += 2; }
+    c = v & 1u;                       if (n >= c) { pos += 1; }
+    return pos;
 }
 
 static __device__ __forceinline__ uint32_t slots_of(int c) { return 256u >> c; }
@@ -199,6 +219,38 @@ static __device__ __noinline__ int bsem_wait_impl(uint64_t* s, uint32_t N, uint3
             w = a_add(s, (uint64_t)N) + (uint64_t)N;                                            // R -= N
         }
     }
+#if GA_OPT_LOAD_GATED
+    // Optimistic form, load-gated: each decision is taken on a plain load and
+    // applied with ONE fetch-add; C is only decremented when the load showed
+    // enough units, so a hot order semaphore is not disturbed by waiters.
+    //   load C >= N          -> fetch-add C -= N (ACQUIRED unless raced: give back)
+    //   load C + D < N       -> fetch-add E += B - N: GROW
+    //   otherwise            -> fetch-add R += N, spin (R-2), R -= N, re-decide
+    // A stale load can only over-produce (an extra split stays inside the tree)
+    // or send a reserved waiter straight back to re-decide; it never over-grants.
+    w = ld_rlx(s);
+    for (;;) {
+        if (sem_C(w) >= (int32_t)N) {
+            uint64_t old = a_add(s, (uint64_t)0 - dn);
+            if (sem_C(old) >= (int32_t)N) return kAcquired;
+            w = a_add(s, dn) + dn;
+            continue;
+        }
+        if ((int64_t)sem_C(w) + sem_D(w) < (int64_t)N) {
+            a_add(s, (uint64_t)(B - N));                                                        // E += B - N
+            return kGrow;
+        }
+        w = a_add(s, (uint64_t)0 - (uint64_t)N) - (uint64_t)N;                                  // R += N
+        uint32_t ns = 32;
+        while (sem_C(w) < (int32_t)N && (int64_t)sem_C(w) + sem_D(w) >= 0) {                    // R-2
+            spin();
+            __nanosleep(ns);
+            if (ns < GA_TREE_SPIN_CAP) ns <<= 1;
+            w = ld_rlx(s);
+        }
+        w = a_add(s, (uint64_t)N) + (uint64_t)N;                                                // R -= N
+    }
+#else
     // Optimistic form: one fetch-add C -= N decides on the pre-image.
     //   pre C >= N           -> ACQUIRED (one atomic, no retry)
     //   pre C + D < N        -> GROW: give C back, E += B - N
@@ -218,11 +270,12 @@ static __device__ __noinline__ int bsem_wait_impl(uint64_t* s, uint32_t N, uint3
         while (sem_C(w) < (int32_t)N && (int64_t)sem_C(w) + sem_D(w) >= 0) {                    // R-2
             spin();
             __nanosleep(ns);
-            if (ns < 256) ns <<= 1;                         // a split lands within a few round trips
+            if (ns < GA_TREE_SPIN_CAP) ns <<= 1;
             w = ld_rlx(s);
         }
         a_add(s, (uint64_t)N);                                                                  // R -= N
     }
+#endif
 }
 // Alg. 1.  Returns kAcquired (0) or kGrow (-1; the caller must
 // produce B units, keep N and signal(B - N, B - N), or signal(0, B - N) on
@@ -346,8 +399,12 @@ static __device__ __forceinline__ void tree_publish(const ga_desc* h, int n, uin
 static __device__ __noinline__ uint64_t tree_claim_word(const ga_desc* h, int n, int need, uint32_t seed, uint64_t* wj) {
     HB3 b = level_hb(h, n);
     uint32_t ns = 32;
+#if GA_LVL_HINT
     int64_t j = ld_rlx32(&h->lvl_hint[n]);                   // the last word a claim succeeded in
     if (j >= b.n0 || ld_rlx(&b.w0[j]) == 0) j = -1;
+#else
+    int64_t j = -1;
+#endif
     for (;;) {
         if (j < 0) j = hb3_find(b, seed);
         if (j >= 0) {
@@ -358,7 +415,9 @@ static __device__ __noinline__ uint64_t tree_claim_word(const ga_desc* h, int n,
                 uint64_t got = old & m;
                 if (old != 0 && (old & ~m) == 0) hb3_up_clear(b, (uint32_t)j);
                 if (got) {
+#if GA_LVL_HINT
                     if ((old & ~m) && ld_rlx32(&h->lvl_hint[n]) != (uint32_t)j) st_rlx32(&h->lvl_hint[n], (uint32_t)j);
+#endif
                     *wj = (uint64_t)j;
                     return got;
                 }
@@ -404,7 +463,7 @@ static __device__ __noinline__ void tree_free(const ga_desc* h, int n, uint64_t 
         bool root = (n >= (int)h->L) || !node_inside(h, n, x ^ 1);
         uint64_t w = ld_rlx(wp);
         if (!root && (w & yb)) {
-            if (bsem_trywait_direct(tsem_ptr(h, n), 1)) {
+            if (GA_MERGE_PRELOAD ? bsem_trywait(tsem_ptr(h, n), 1) : bsem_trywait_direct(tsem_ptr(h, n), 1)) {
                 uint64_t old = a_and(wp, ~yb);
                 if (old & yb) {                               // merged: free the parent at n + 1
                     if (old == yb) hb3_up_clear(b, (uint32_t)(x >> 6));
@@ -827,48 +886,58 @@ static __device__ __noinline__ uint64_t bin_malloc_lane(const ga_desc* h, uint32
     return kNull;
 }
 
-// ---- bins: collective claim of one slot per lane (units already acquired) ----
-// Lanes spread over the chunk's non-full pages by their rank (each thread walks
-// the number of elements its index dictates), lanes that picked
-// the same page regroup and that page gets ONE atomicOr for all of them.
-static __device__ __noinline__ uint64_t bin_claim_collective(const ga_desc* h, unsigned grp, uint32_t A, int c) {
+// ---- warp-wide collective steps -------------------------------------------------
+// A warp's lanes are grouped by size class (one group per class, mask `grp`).
+// The collective steps below run for ALL groups of the warp at once: every
+// warp-sync intrinsic uses the mask of all participating lanes (`live`), each
+// lane reading from its own group's leader, and __syncwarp(live) reconverges
+// the warp before each atomic, so the groups' atomics issue in the same
+// instruction instead of one group after another.
+
+// ---- bins: one slot per lane; every group of `live` holds its units ------------
+// Lanes spread over the chunk's non-full pages by their rank in the group (each
+// thread walks the number of elements its index dictates); lanes
+// that picked the same page regroup, and that page gets ONE atomicOr for all of them.
+static __device__ __noinline__ uint64_t bin_claim_collective(const ga_desc* h, unsigned live, unsigned grp, uint32_t A, int c) {
     const uint32_t lane = lane_id();
     const uint32_t per_page = slots_of(c) < 64 ? slots_of(c) : 64;
     const uint64_t csz = 16ull << c;
     uint64_t my = kNull;
-    unsigned unsat = grp;                                   // lanes still without a slot (this lane included)
     for (;;) {
-        const int L = __ffs(unsat) - 1;
+        const unsigned mine = live & grp;                        // my group's lanes still without a slot
+        const int L = __ffs(mine) - 1;
         uint64_t ch = 0, m = 0;
         if ((int)lane == L) ch = bin_find_chunk(h, A, c, &m);
-        ch = __shfl_sync(unsat, ch, L);
-        m = __shfl_sync(unsat, m, L);
-        const uint32_t q = __popc(unsat & lanemask_lt());
+        __syncwarp(live);
+        ch = __shfl_sync(live, ch, L);
+        m = __shfl_sync(live, m, L);
+        const uint32_t q = __popc(mine & lanemask_lt());
         const uint32_t np = __popcll(m);
         const uint64_t page = ch * kChunkPages + nth_set(m, (q / per_page) % np);
-        const unsigned pg = __match_any_sync(unsat, page);
+        const unsigned pg = __match_any_sync(live, (page << 3) | (uint64_t)c);
         const int pl = __ffs(pg) - 1;
         uint64_t got = 0;
         int wi = 0;
         if ((int)lane == pl) got = bin_claim_page(h, page, A, c, __popc(pg), &wi);
-        got = __shfl_sync(pg, got, pl);
-        wi = __shfl_sync(pg, wi, pl);
+        __syncwarp(live);
+        got = __shfl_sync(live, got, pl);
+        wi = __shfl_sync(live, wi, pl);
         const uint32_t pr = __popc(pg & lanemask_lt());
         if (pr < (uint32_t)__popcll(got)) my = (page << kPageShift) + (uint64_t)(wi * 64 + nth_set(got, pr)) * csz;
-        unsat = __ballot_sync(unsat, my == kNull);
-        if (my != kNull) break;                             // a satisfied lane leaves the group
+        live = __ballot_sync(live, my == kNull);
+        if (my != kNull) break;                                  // a served lane leaves
     }
     return my;
 }
 
-// ---- bins: collective growth (class semaphore said GROW for the group) ------
-// The leader accounts ceil(N/slots) pages on the arena page semaphore and
-// tracks them one chunk at a time (one atomicOr claims several pages: the
-// collective chunk-list split of P:L1282-1292); every lane computes its page
-// and slot, the first lane of each page initialises that bin, then the leader
-// publishes the spare slots with one signal.  Returns kNull for every lane if
-// the group could not grow (the caller degrades to per-lane waits).
-static __device__ __noinline__ uint64_t bin_grow_collective(const ga_desc* h, unsigned grp, uint32_t A, int c) {
+// ---- bins: collective growth (the class semaphore said GROW for these groups) ----
+// Each group's leader accounts ceil(N/slots) pages on the arena page semaphore
+// and tracks them one chunk at a time (one atomicOr claims several pages: the
+// collective chunk-list split of P:L1282-1292); each lane computes its page and
+// slot, the first lane of each page initialises that bin, then the leader
+// publishes the spare slots with one signal.  A group that cannot grow returns
+// kNull on every lane (the caller degrades it to per-lane waits).
+static __device__ __noinline__ uint64_t bin_grow_collective(const ga_desc* h, unsigned live, unsigned grp, uint32_t A, int c) {
     const uint32_t lane = lane_id();
     const int leader = __ffs(grp) - 1;
     const uint32_t N = __popc(grp), rank = __popc(grp & lanemask_lt());
@@ -885,7 +954,7 @@ static __device__ __noinline__ uint64_t bin_grow_collective(const ga_desc* h, un
             int64_t nc = chunk_acquire(h, A, k);
             if (nc < 0) {
                 bsem_signal(psem_ptr(h, A), 0, kChunkPages - k);
-                bsem_signal(sem_ptr(h, A, c), 0, Bp - N);
+                bsem_signal(sem_ptr(h, A, c), 0, Bp - N);                   // failure signal
                 mode = -1;
             } else {
                 bsem_signal(psem_ptr(h, A), kChunkPages - k, kChunkPages - k);
@@ -893,14 +962,17 @@ static __device__ __noinline__ uint64_t bin_grow_collective(const ga_desc* h, un
             }
         }
     }
-    mode = __shfl_sync(grp, mode, leader);
+    __syncwarp(live);
+    mode = __shfl_sync(live, mode, leader);
+    live = __ballot_sync(live, mode >= 0);
     if (mode < 0) return kNull;
     uint32_t served = 0, pages_left = k;
     uint64_t last_page = 0;
-    while (pages_left) {
+    for (;;) {
         if (mode == 0 && (int)lane == leader) pm = page_claim(h, A, (int)pages_left, &ch);
-        ch = __shfl_sync(grp, ch, leader);
-        pm = __shfl_sync(grp, pm, leader);
+        __syncwarp(live);
+        ch = __shfl_sync(live, ch, leader);
+        pm = __shfl_sync(live, pm, leader);
         const uint32_t np = __popcll(pm);
         const uint32_t cap = np * slots;
         if (rank >= served && rank < served + cap) {
@@ -916,23 +988,26 @@ static __device__ __noinline__ uint64_t bin_grow_collective(const ga_desc* h, un
         served += cap < N - served ? cap : N - served;
         pages_left -= np;
         mode = 0;
+        const bool done = pages_left == 0;                                   // uniform within the group
+        live = __ballot_sync(live, !done);
+        if (done) break;
     }
-    __syncwarp(grp);
+    __syncwarp(grp);                                                         // every bin of the group is initialised
     if ((int)lane == leader) {
         stat_add(h, kStatBinGrow, k);
         st_rlx32(&h->hint[A * kNcls + c], (uint32_t)last_page);
-        bsem_signal(sem_ptr(h, A, c), Bp - N, Bp - N);                      // release: bins are initialised
+        bsem_signal(sem_ptr(h, A, c), Bp - N, Bp - N);                      // release the spare slots
     }
     return my;
 }
 
-// ---- TBuddy, group path -------------------------------------------------------
-// One bulk wait of N units per order for the group (batch 2, B' = 2*ceil(N/2));
+// ---- TBuddy, groups of `live` at once ------------------------------------------
+// One bulk wait of N units per order for each group (batch 2, B' = 2*ceil(N/2));
 // on GROW the group climbs with N_{k+1} = ceil(N_k / 2), claims N_m nodes at the
 // granting level m and splits them down: each claimed node serves 2^(m-o)
-// lanes, the unused right parts of the last node are published.  Returns kNull
-// for every lane if the tree could not serve the whole group.
-static __device__ __noinline__ uint64_t tree_malloc_group(const ga_desc* h, unsigned grp, int o) {
+// lanes, the unused right parts of the last node are published by the group's
+// lanes in parallel.  A group the tree cannot serve returns kNull on every lane.
+static __device__ __noinline__ uint64_t tree_malloc_collective(const ga_desc* h, unsigned live, unsigned grp, int o) {
     const uint32_t lane = lane_id();
     const int leader = __ffs(grp) - 1;
     const uint32_t N = __popc(grp), rank = __popc(grp & lanemask_lt());
@@ -943,7 +1018,7 @@ static __device__ __noinline__ uint64_t tree_malloc_group(const ga_desc* h, unsi
         for (int attempt = 0;; attempt++) {
             m = o; Nm = N;
             for (;;) {
-                if (m > (int)h->L) {                         // nothing to grow from: retract every E
+                if (m > (int)h->L) {                                        // nothing to grow from: retract every E
                     uint32_t nk = N;
                     for (int k = o; k < m; k++) { bsem_signal(tsem_ptr(h, k), 0, 2 * ((nk + 1) >> 1) - nk); nk = (nk + 1) >> 1; }
                     m = -1;
@@ -959,34 +1034,33 @@ static __device__ __noinline__ uint64_t tree_malloc_group(const ga_desc* h, unsi
             __nanosleep(ns); if (ns < 8192) ns <<= 1;
         }
     }
-    m = __shfl_sync(grp, m, leader);
+    __syncwarp(live);
+    m = __shfl_sync(live, m, leader);
+    Nm = __shfl_sync(live, Nm, leader);
+    live = __ballot_sync(live, m >= 0);
     if (m < 0) return kNull;
-    Nm = __shfl_sync(grp, Nm, leader);
     const int s = m - o;
     uint64_t my = kNull;
     uint32_t served = 0;
-    uint32_t seed = scatter_seed();
-    while (served < N) {
+    const uint32_t seed = scatter_seed();
+    for (;;) {
         uint64_t wj = 0, got = 0;
         if ((int)lane == leader) got = tree_claim_word(h, m, (int)(Nm - (served >> s)), seed, &wj);
-        wj = __shfl_sync(grp, wj, leader);
-        got = __shfl_sync(grp, got, leader);
-        {
-            const uint32_t nn = __popcll(got), rem = N - served;
-            if ((nn << s) >= rem && s > 0) {
-                // the last node is split: its unused right parts [pos, 2^s) decompose into
-                // one aligned block per set bit j of the running position (E at each level
-                // o + j); the group's lanes publish them in parallel, lane q doing level o + q
-                const uint64_t xlast = wj * 64 + (63 - __clzll((long long)got));
-                const uint64_t keep = rem - ((nn - 1) << s);
-                for (uint32_t j = rank; j < (uint32_t)s; j += N) {
-                    // running position before level j = keep rounded up to a multiple of 2^j
-                    const uint64_t pj = (keep + (1ull << j) - 1) & ~((1ull << j) - 1);
-                    if ((pj >> j) & 1) tree_publish(h, o + (int)j, ((xlast << s) + pj) >> j, 1);
-                }
+        __syncwarp(live);
+        wj = __shfl_sync(live, wj, leader);
+        got = __shfl_sync(live, got, leader);
+        const uint32_t nn = __popcll(got), rem = N - served, cap = nn << s;
+        if ((nn << s) >= rem && s > 0) {
+            // the last node is split: its unused right parts decompose into one aligned
+            // block per level o + j where the running position (keep rounded up to 2^j)
+            // has bit j set -- the E each level's GROW promised; lanes publish in parallel
+            const uint64_t xlast = wj * 64 + (63 - __clzll((long long)got));
+            const uint64_t keep = rem - ((nn - 1) << s);
+            for (uint32_t j = rank; j < (uint32_t)s; j += N) {
+                const uint64_t pj = (keep + (1ull << j) - 1) & ~((1ull << j) - 1);
+                if ((pj >> j) & 1) tree_publish(h, o + (int)j, ((xlast << s) + pj) >> j, 1);
             }
         }
-        const uint32_t cap = (uint32_t)__popcll(got) << s;
         if (rank >= served && rank < served + cap) {
             const uint32_t r = rank - served;
             const uint64_t x = wj * 64 + nth_set(got, r >> s);
@@ -994,7 +1068,10 @@ static __device__ __noinline__ uint64_t tree_malloc_group(const ga_desc* h, unsi
             st_rlx32(&h->kind[pg], kKindTree | (uint32_t)o);
             my = pg << kPageShift;
         }
-        served += cap < N - served ? cap : N - served;
+        served += cap < rem ? cap : rem;
+        const bool done = served >= N;                                       // uniform within the group
+        live = __ballot_sync(live, !done);
+        if (done) break;
     }
     return my;
 }
@@ -1004,24 +1081,30 @@ static __device__ __noinline__ uint64_t ga_malloc_off(const ga_desc* h, uint64_t
     const unsigned act = __activemask();
     const int key = size_key(h, n);
     const unsigned grp = __match_any_sync(act, key);
+    const unsigned bins = __ballot_sync(act, key >= 0 && key < kNcls);
+    const unsigned trees = __ballot_sync(act, key >= kNcls);
     if (key < 0) return kNull;
+    const uint32_t lane = lane_id();
+    const int leader = __ffs(grp) - 1;
     uint64_t my;
     if (key < kNcls) {
         const uint32_t A = arena_of(h);
         const uint32_t N = __popc(grp), slots = slots_of(key);
-        const int leader = __ffs(grp) - 1;
         int r = 0;
-        if ((int)lane_id() == leader)
+        if ((int)lane == leader)                                   // every group's leader at once
             r = bsem_wait(sem_ptr(h, A, key), N, slots * ((N + slots - 1) / slots), ArenaSpin{h, A});
-        r = __shfl_sync(grp, r, leader);
-        my = r == kAcquired ? bin_claim_collective(h, grp, A, key) : bin_grow_collective(h, grp, A, key);
-        if (__any_sync(grp, my == kNull)) {                 // R-27: degrade to per-lane waits
-            if ((int)lane_id() == leader) stat_add(h, kStatFallback, 1);
-            if (my == kNull) my = bin_malloc_lane(h, A, key);
+        __syncwarp(bins);
+        r = __shfl_sync(bins, r, leader);
+        const unsigned acq = __ballot_sync(bins, r == kAcquired);
+        if (r == kAcquired) my = bin_claim_collective(h, acq, grp, A, key);
+        else my = bin_grow_collective(h, bins & ~acq, grp, A, key);
+        if (my == kNull) {                                         // R-27: the group degrades to per-lane waits
+            if ((int)lane == leader) stat_add(h, kStatFallback, 1);
+            my = bin_malloc_lane(h, A, key);
         }
     } else {
         const int o = key - kNcls;
-        my = tree_malloc_group(h, grp, o);
+        my = tree_malloc_collective(h, trees, grp, o);
         if (my == kNull) {
             int64_t x = tree_alloc_one_retry(h, o);
             if (x >= 0) {
@@ -1048,7 +1131,7 @@ static __device__ __noinline__ void ga_free_off(const ga_desc* h, uint64_t off) 
     const unsigned bins = __ballot_sync(act, is_bin);
     const unsigned trees = __ballot_sync(act, is_tree);
     if (is_tree) {
-        int n = (int)(k & 0xFF);                               // order from the page kind (R-18)
+        int n = (int)(k & 0xFF);                                   // order from the page kind (R-18)
         uint64_t x = p >> n;
         st_rlx32(&h->kind[p], 0);
         fence();
@@ -1077,12 +1160,13 @@ static __device__ __noinline__ void ga_free_off(const ga_desc* h, uint64_t off) 
     const unsigned g1 = __match_any_sync(bins, (p << 2) | (uint64_t)w);
     const uint64_t bit = 1ull << (slot & 63);
     const uint64_t mask = ((uint64_t)__reduce_or_sync(g1, (uint32_t)(bit >> 32)) << 32) | __reduce_or_sync(g1, (uint32_t)bit);
-    if ((int)lane_id() == __ffs(g1) - 1) {
+    __syncwarp(bins);
+    if ((int)lane_id() == __ffs(g1) - 1) {                         // every word's leader at once
         uint64_t* bw = page_bits(h, p);
         const uint64_t old = a_and(&bw[w], ~mask);
         const uint64_t v = valid_mask(c, w);
-        if ((old | ~v) == ~0ull) nonfull_set(h, p, c, A);     // the word was full: bin back in the list
-        if (((old & ~mask) & v) == 0) {                        // this word is empty: is the bin?
+        if ((old | ~v) == ~0ull) nonfull_set(h, p, c, A);         // the word was full: bin back in the list
+        if (((old & ~mask) & v) == 0) {                            // this word is empty: is the bin?
             uint64_t ww[4];
             ld_bitmap(bw, ww);
             bool empty = true;
