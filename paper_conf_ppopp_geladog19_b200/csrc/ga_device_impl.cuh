@@ -930,137 +930,133 @@ static __device__ __noinline__ uint64_t bin_claim_collective(const ga_desc* h, u
     return my;
 }
 
-// ---- bins: collective growth (the class semaphore said GROW for these groups) ----
-// Each group's leader accounts ceil(N/slots) pages on the arena page semaphore
-// and tracks them one chunk at a time (one atomicOr claims several pages: the
-// collective chunk-list split of P:L1282-1292); each lane computes its page and
-// slot, the first lane of each page initialises that bin, then the leader
-// publishes the spare slots with one signal.  A group that cannot grow returns
-// kNull on every lane (the caller degrades it to per-lane waits).
-static __device__ __noinline__ uint64_t bin_grow_collective(const ga_desc* h, unsigned live, unsigned grp, uint32_t A, int c) {
-    const uint32_t lane = lane_id();
-    const int leader = __ffs(grp) - 1;
-    const uint32_t N = __popc(grp), rank = __popc(grp & lanemask_lt());
+// ---- bins: growth, done by the group's leader before any warp-wide sync ----------
+// (a leader blocked in a semaphore wait may be waiting for this very production
+// in another warp, so production must never wait on a warp barrier).  The leader
+// accounts ceil(N/slots) pages on the arena page semaphore, tracks them one chunk
+// at a time (one atomicOr claims several pages: the collective chunk-list split
+// of P:L1282-1292), initialises every new bin (the group keeps the first N
+// slots) and publishes the spare slots with one signal.  The pages are recorded
+// as (chunk, page mask) runs for the lanes.  Returns the number of runs, 0 on
+// failure (every E retracted).
+constexpr int kMaxRuns = 16;
+static __device__ __noinline__ int bin_grow_leader(const ga_desc* h, uint32_t A, int c, uint32_t N,
+                                                   uint64_t* run_ch, uint64_t* run_pm) {
     const uint32_t slots = slots_of(c);
     const uint32_t Bp = slots * ((N + slots - 1) / slots);                 // R-8
     const uint32_t k = Bp / slots;
-    const uint64_t csz = 16ull << c;
-    uint64_t my = kNull;
-    int mode = 0;                                                            // 0 claim pages, 1 fresh chunk, -1 fail
-    uint64_t ch = 0, pm = 0;
-    if ((int)lane == leader) {
-        if (bsem_wait(psem_ptr(h, A), k, kChunkPages, ArenaSpin{h, A}) == kGrow) {
-            reclaim_arena(h, A, -1, kReclaimKeep);                           // delegated work first
-            int64_t nc = chunk_acquire(h, A, k);
-            if (nc < 0) {
-                bsem_signal(psem_ptr(h, A), 0, kChunkPages - k);
-                bsem_signal(sem_ptr(h, A, c), 0, Bp - N);                   // failure signal
-                mode = -1;
-            } else {
-                bsem_signal(psem_ptr(h, A), kChunkPages - k, kChunkPages - k);
-                mode = 1; ch = (uint64_t)nc; pm = k >= 64 ? ~0ull : ((1ull << k) - 1);
-            }
-        }
-    }
-    __syncwarp(live);
-    mode = __shfl_sync(live, mode, leader);
-    live = __ballot_sync(live, mode >= 0);
-    if (mode < 0) return kNull;
-    uint32_t served = 0, pages_left = k;
+    int nruns = 0;
+    uint32_t pages_left = k, left = N;
     uint64_t last_page = 0;
-    for (;;) {
-        if (mode == 0 && (int)lane == leader) pm = page_claim(h, A, (int)pages_left, &ch);
-        __syncwarp(live);
-        ch = __shfl_sync(live, ch, leader);
-        pm = __shfl_sync(live, pm, leader);
-        const uint32_t np = __popcll(pm);
-        const uint32_t cap = np * slots;
-        if (rank >= served && rank < served + cap) {
-            const uint32_t r = rank - served;
-            const uint64_t p = ch * kChunkPages + nth_set(pm, r / slots);
-            my = (p << kPageShift) + (uint64_t)(r % slots) * csz;
-            if (r % slots == 0) {
-                const uint32_t left = N - served - (r / slots) * slots;
-                bin_init(h, p, A, c, left < slots ? left : slots);
-            }
+    if (bsem_wait(psem_ptr(h, A), k, kChunkPages, ArenaSpin{h, A}) == kGrow) {
+        reclaim_arena(h, A, -1, kReclaimKeep);                              // delegated work first
+        int64_t nc = chunk_acquire(h, A, k);
+        if (nc < 0) {
+            bsem_signal(psem_ptr(h, A), 0, kChunkPages - k);
+            bsem_signal(sem_ptr(h, A, c), 0, Bp - N);
+            return 0;
         }
-        last_page = ch * kChunkPages + nth_set(pm, np - 1);
-        served += cap < N - served ? cap : N - served;
-        pages_left -= np;
-        mode = 0;
-        const bool done = pages_left == 0;                                   // uniform within the group
-        live = __ballot_sync(live, !done);
-        if (done) break;
+        bsem_signal(psem_ptr(h, A), kChunkPages - k, kChunkPages - k);
+        run_ch[0] = (uint64_t)nc;
+        run_pm[0] = k >= 64 ? ~0ull : ((1ull << k) - 1);
+        nruns = 1;
+        pages_left = 0;
     }
-    __syncwarp(grp);                                                         // every bin of the group is initialised
-    if ((int)lane == leader) {
-        stat_add(h, kStatBinGrow, k);
-        st_rlx32(&h->hint[A * kNcls + c], (uint32_t)last_page);
-        bsem_signal(sem_ptr(h, A, c), Bp - N, Bp - N);                      // release the spare slots
+    while (pages_left) {
+        uint64_t ch;
+        uint64_t pm = page_claim(h, A, (int)pages_left, &ch);
+        run_ch[nruns] = ch; run_pm[nruns] = pm; nruns++;
+        pages_left -= __popcll(pm);
     }
-    return my;
+    for (int i = 0; i < nruns; i++) {
+        uint64_t pm = run_pm[i];
+        while (pm) {
+            uint64_t p = run_ch[i] * kChunkPages + (uint64_t)(__ffsll((long long)pm) - 1);
+            pm &= pm - 1;
+            bin_init(h, p, A, c, left < slots ? left : slots);
+            left -= left < slots ? left : slots;
+            last_page = p;
+        }
+    }
+    stat_add(h, kStatBinGrow, k);
+    st_rlx32(&h->hint[A * kNcls + c], (uint32_t)last_page);
+    bsem_signal(sem_ptr(h, A, c), Bp - N, Bp - N);                          // release the spare slots
+    return nruns;
 }
 
-// ---- TBuddy, groups of `live` at once ------------------------------------------
-// One bulk wait of N units per order for each group (batch 2, B' = 2*ceil(N/2));
-// on GROW the group climbs with N_{k+1} = ceil(N_k / 2), claims N_m nodes at the
-// granting level m and splits them down: each claimed node serves 2^(m-o)
-// lanes, the unused right parts of the last node are published by the group's
-// lanes in parallel.  A group the tree cannot serve returns kNull on every lane.
-static __device__ __noinline__ uint64_t tree_malloc_collective(const ga_desc* h, unsigned live, unsigned grp, int o) {
+// ---- TBuddy: the leader's climb (Alg. 1 per order) ------------------
+// One bulk wait of N units per order (batch 2, B' = 2*ceil(N/2)); on GROW the
+// group climbs with N_{k+1} = ceil(N_k / 2) until an order m grants N_m nodes.
+// If the last node is only partly used, the leader claims it first and
+// publishes its unused right parts right away -- the E each level's GROW
+// promised -- so no waiter depends on work behind a warp barrier.
+// Returns m (or -1 after retracting every E); *xpart = the partly used node.
+static __device__ __noinline__ int tree_climb_leader(const ga_desc* h, int o, uint32_t N, uint32_t* Nm_out, uint64_t* xpart) {
+    int m = o;
+    uint32_t Nm = N;
+    uint32_t ns = 128;
+    for (int attempt = 0;; attempt++) {
+        m = o; Nm = N;
+        for (;;) {
+            if (m > (int)h->L) {                                            // nothing to grow from: retract every E
+                uint32_t nk = N;
+                for (int k = o; k < m; k++) { bsem_signal(tsem_ptr(h, k), 0, 2 * ((nk + 1) >> 1) - nk); nk = (nk + 1) >> 1; }
+                m = -1;
+                break;
+            }
+            if (bsem_wait_fast(tsem_ptr(h, m), Nm, 2 * ((Nm + 1) >> 1), NoSpin()) == kAcquired) break;
+            Nm = (Nm + 1) >> 1;
+            m++;
+        }
+        // No false resource starvation: while splits are in flight
+        // (cold start) or units are visible at some order >= o, re-climb
+        if (m >= 0 || attempt >= 8 || !tree_has_supply(h, o, attempt < 2)) break;
+        __nanosleep(ns); if (ns < 8192) ns <<= 1;
+    }
+    *Nm_out = Nm;
+    *xpart = kNull;
+    const int s = m - o;
+    if (m >= 0 && s > 0 && (N & ((1u << s) - 1))) {
+        uint64_t wj;
+        uint64_t got = tree_claim_word(h, m, 1, scatter_seed(), &wj);
+        const uint64_t x = wj * 64 + (uint64_t)(__ffsll((long long)got) - 1);
+        const uint64_t keep = N & ((1u << s) - 1);                          // lanes served by x
+        for (int j = 0; j < s; j++) {
+            const uint64_t pj = (keep + (1ull << j) - 1) & ~((1ull << j) - 1);
+            if ((pj >> j) & 1) tree_publish(h, o + j, ((x << s) + pj) >> j, 1);
+        }
+        *xpart = x;
+    }
+    return m;
+}
+
+// ---- TBuddy: full nodes claimed for all groups of `live` at once ---------------
+// (only claims: the units are held, nothing is produced here)
+static __device__ __noinline__ uint64_t tree_claim_collective(const ga_desc* h, unsigned live, unsigned grp, int o, int m,
+                                                              uint32_t Nm, uint64_t xpart) {
     const uint32_t lane = lane_id();
     const int leader = __ffs(grp) - 1;
     const uint32_t N = __popc(grp), rank = __popc(grp & lanemask_lt());
-    int m = o;
-    uint32_t Nm = N;
-    if ((int)lane == leader) {
-        uint32_t ns = 128;
-        for (int attempt = 0;; attempt++) {
-            m = o; Nm = N;
-            for (;;) {
-                if (m > (int)h->L) {                                        // nothing to grow from: retract every E
-                    uint32_t nk = N;
-                    for (int k = o; k < m; k++) { bsem_signal(tsem_ptr(h, k), 0, 2 * ((nk + 1) >> 1) - nk); nk = (nk + 1) >> 1; }
-                    m = -1;
-                    break;
-                }
-                if (bsem_wait_fast(tsem_ptr(h, m), Nm, 2 * ((Nm + 1) >> 1), NoSpin()) == kAcquired) break;
-                Nm = (Nm + 1) >> 1;
-                m++;
-            }
-            // No false resource starvation: while splits are in flight
-            // (cold start) or units are visible at some order >= o, re-climb
-            if (m >= 0 || attempt >= 8 || !tree_has_supply(h, o, attempt < 2)) break;
-            __nanosleep(ns); if (ns < 8192) ns <<= 1;
-        }
-    }
-    __syncwarp(live);
-    m = __shfl_sync(live, m, leader);
-    Nm = __shfl_sync(live, Nm, leader);
-    live = __ballot_sync(live, m >= 0);
-    if (m < 0) return kNull;
     const int s = m - o;
+    const uint32_t nfull = xpart == kNull ? Nm : Nm - 1;                   // nodes serving 2^s lanes each
+    const uint32_t full_lanes = nfull << s;
     uint64_t my = kNull;
-    uint32_t served = 0;
+    if (rank >= full_lanes) {                                              // lanes of the partly used node
+        const uint64_t pg = ((xpart << s) + (rank - full_lanes)) << o;
+        st_rlx32(&h->kind[pg], kKindTree | (uint32_t)o);
+        my = pg << kPageShift;
+    }
+    live = __ballot_sync(live, nfull > 0);
+    if (nfull == 0) return my;
+    uint32_t served = 0;                                                   // lanes served from full nodes
     const uint32_t seed = scatter_seed();
     for (;;) {
         uint64_t wj = 0, got = 0;
-        if ((int)lane == leader) got = tree_claim_word(h, m, (int)(Nm - (served >> s)), seed, &wj);
+        if ((int)lane == leader) got = tree_claim_word(h, m, (int)(nfull - (served >> s)), seed, &wj);
         __syncwarp(live);
         wj = __shfl_sync(live, wj, leader);
         got = __shfl_sync(live, got, leader);
-        const uint32_t nn = __popcll(got), rem = N - served, cap = nn << s;
-        if ((nn << s) >= rem && s > 0) {
-            // the last node is split: its unused right parts decompose into one aligned
-            // block per level o + j where the running position (keep rounded up to 2^j)
-            // has bit j set -- the E each level's GROW promised; lanes publish in parallel
-            const uint64_t xlast = wj * 64 + (63 - __clzll((long long)got));
-            const uint64_t keep = rem - ((nn - 1) << s);
-            for (uint32_t j = rank; j < (uint32_t)s; j += N) {
-                const uint64_t pj = (keep + (1ull << j) - 1) & ~((1ull << j) - 1);
-                if ((pj >> j) & 1) tree_publish(h, o + (int)j, ((xlast << s) + pj) >> j, 1);
-            }
-        }
+        const uint32_t cap = (uint32_t)__popcll(got) << s;
         if (rank >= served && rank < served + cap) {
             const uint32_t r = rank - served;
             const uint64_t x = wj * 64 + nth_set(got, r >> s);
@@ -1068,15 +1064,17 @@ static __device__ __noinline__ uint64_t tree_malloc_collective(const ga_desc* h,
             st_rlx32(&h->kind[pg], kKindTree | (uint32_t)o);
             my = pg << kPageShift;
         }
-        served += cap < rem ? cap : rem;
-        const bool done = served >= N;                                       // uniform within the group
+        served += cap;
+        const bool done = served >= full_lanes;                              // uniform within the group
         live = __ballot_sync(live, !done);
         if (done) break;
     }
+    (void)N;
     return my;
 }
 
 // ---- the entry points ---------------------------------------------------------
+enum { kRGrown = 2, kRFailed = 3 };
 static __device__ __noinline__ uint64_t ga_malloc_off(const ga_desc* h, uint64_t n) {
     const unsigned act = __activemask();
     const int key = size_key(h, n);
@@ -1086,25 +1084,58 @@ static __device__ __noinline__ uint64_t ga_malloc_off(const ga_desc* h, uint64_t
     if (key < 0) return kNull;
     const uint32_t lane = lane_id();
     const int leader = __ffs(grp) - 1;
-    uint64_t my;
+    const uint32_t N = __popc(grp), rank = __popc(grp & lanemask_lt());
+    uint64_t my = kNull;
     if (key < kNcls) {
         const uint32_t A = arena_of(h);
-        const uint32_t N = __popc(grp), slots = slots_of(key);
-        int r = 0;
-        if ((int)lane == leader)                                   // every group's leader at once
+        const uint32_t slots = slots_of(key);
+        int r = 0, nruns = 0;
+        uint64_t run_ch[kMaxRuns], run_pm[kMaxRuns];
+        if ((int)lane == leader) {                                 // every group's leader at once
             r = bsem_wait(sem_ptr(h, A, key), N, slots * ((N + slots - 1) / slots), ArenaSpin{h, A});
-        __syncwarp(bins);
+            if (r == kGrow) {
+                nruns = bin_grow_leader(h, A, key, N, run_ch, run_pm);
+                r = nruns ? kRGrown : kRFailed;
+            }
+        }
+        __syncwarp(bins);                                          // all production of this warp is done
         r = __shfl_sync(bins, r, leader);
         const unsigned acq = __ballot_sync(bins, r == kAcquired);
         if (r == kAcquired) my = bin_claim_collective(h, acq, grp, A, key);
-        else my = bin_grow_collective(h, bins & ~acq, grp, A, key);
+        else if (r == kRGrown) {
+            // hand the new slots out: rank -> (run, page, slot), group-local
+            nruns = __shfl_sync(grp, nruns, leader);
+            uint32_t base = 0;
+            const uint64_t csz = 16ull << key;
+            for (int i = 0; i < nruns; i++) {
+                uint64_t ch = 0, pm = 0;
+                if ((int)lane == leader) { ch = run_ch[i]; pm = run_pm[i]; }
+                ch = __shfl_sync(grp, ch, leader);
+                pm = __shfl_sync(grp, pm, leader);
+                const uint32_t cap = (uint32_t)__popcll(pm) * slots;
+                if (rank >= base && rank < base + cap) {
+                    const uint32_t q = rank - base;
+                    my = ((ch * kChunkPages + nth_set(pm, q / slots)) << kPageShift) + (uint64_t)(q % slots) * csz;
+                }
+                base += cap;
+            }
+        }
         if (my == kNull) {                                         // R-27: the group degrades to per-lane waits
             if ((int)lane == leader) stat_add(h, kStatFallback, 1);
             my = bin_malloc_lane(h, A, key);
         }
     } else {
         const int o = key - kNcls;
-        my = tree_malloc_collective(h, trees, grp, o);
+        int m = -1;
+        uint32_t Nm = 0;
+        uint64_t xpart = kNull;
+        if ((int)lane == leader) m = tree_climb_leader(h, o, N, &Nm, &xpart);
+        __syncwarp(trees);                                         // every split of this warp is published
+        m = __shfl_sync(trees, m, leader);
+        Nm = __shfl_sync(trees, Nm, leader);
+        xpart = __shfl_sync(trees, xpart, leader);
+        const unsigned ok = __ballot_sync(trees, m >= 0);
+        if (m >= 0) my = tree_claim_collective(h, ok, grp, o, m, Nm, xpart);
         if (my == kNull) {
             int64_t x = tree_alloc_one_retry(h, o);
             if (x >= 0) {
