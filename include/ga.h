@@ -73,6 +73,7 @@ typedef struct ga_desc {
     uint64_t lvl_off[48];     /* word offset of level n in avail                        */
     uint32_t lvl_words[48];   /* u64 words of level n's availability bits               */
     uint32_t* lvl_hint;       /* [48] last level-n word a claim succeeded in            */
+    uint64_t* dbg;            /* GA_DEBUG builds: host-mapped stuck-spin records (or 0) */
 } ga_desc;
 
 /* Plain-old-data handle passed BY VALUE to kernels that call ga_malloc /

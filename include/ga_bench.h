@@ -94,6 +94,12 @@ typedef struct {
 } ga_bsem_cfg;
 ga_status ga_bsem_bench(ga_stream_t stream, const ga_bsem_cfg* cfg, uint64_t* sems, uint64_t* out);
 
+/* Debug builds (-DGA_DEBUG=1) only: allocate a host-mapped buffer where spin
+ * loops that run ~2^18 iterations leave (site, sm|warp|lane, a, b) records,
+ * readable while a kernel hangs; *host_records = u64[8 + 4*256], [0] = count.
+ * Other builds return GA_EINVAL. */
+ga_status ga_debug_attach(uint64_t** host_records);
+
 #ifdef __cplusplus
 }
 #endif

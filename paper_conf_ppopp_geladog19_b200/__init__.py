@@ -28,7 +28,7 @@ EXPORTED = ["ga_heap_create", "ga_heap_destroy", "ga_heap_reset", "ga_stats", "g
             "ga_heap_info", "ga_layout", "ga_heap_quiesce", "ga_heap_snapshot", "ga_reserved_pages",
             "ga_status_str", "ga_trace_phase", "ga_trace_timed", "ga_trace_timed_host",
             "ga_cuda_set_heap_limit", "ga_cuda_trace_phase", "ga_cuda_trace_timed",
-            "ga_kernel_info", "ga_l2_atomic_bench", "ga_bsem_bench"]
+            "ga_kernel_info", "ga_l2_atomic_bench", "ga_bsem_bench", "ga_debug_attach"]
 
 
 class GaError(RuntimeError):
@@ -94,6 +94,7 @@ def lib():
         "ga_kernel_info": [i32, u32, P(i32), P(i32), P(i32)],
         "ga_l2_atomic_bench": [vp, i32, vp, u64, u32, u32, u32, vp],
         "ga_bsem_bench": [vp, P(BsemCfg), vp, vp],
+        "ga_debug_attach": [P(P(u64))],
     }
     for name, args in sig.items():
         f = getattr(L, name)

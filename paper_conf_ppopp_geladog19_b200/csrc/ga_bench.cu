@@ -9,6 +9,7 @@
 #include <cstdint>
 #include <cstdio>
 #include <cstdlib>
+#include <cstring>
 
 #include "ga.h"
 #include "ga_bench.h"
@@ -412,6 +413,23 @@ ga_status ga_l2_atomic_bench(ga_stream_t stream, int pattern, uint64_t* d_buf, u
     if (!d_buf || !d_sink || pattern < 0 || pattern > 5 || n_words < 1184 * 4) return GA_EINVAL;
     k_l2_atomic<<<grid, block, 0, (cudaStream_t)stream>>>(pattern, d_buf, n_words, iters, d_sink, 0u);
     return launched();
+}
+
+ga_status ga_debug_attach(uint64_t** host_records) {
+#if GA_DEBUG
+    if (!host_records) return GA_EINVAL;
+    void* hp = nullptr;
+    if (cudaHostAlloc(&hp, 8 * (8 + 4 * 256), cudaHostAllocMapped) != cudaSuccess) return GA_ENOMEM;
+    memset(hp, 0, 8 * (8 + 4 * 256));
+    void* dp = nullptr;
+    if (cudaHostGetDevicePointer(&dp, hp, 0) != cudaSuccess) return GA_ECUDA;
+    if (cudaMemcpyToSymbol(ga::g_ga_dbg, &dp, sizeof dp) != cudaSuccess) return GA_ECUDA;
+    *host_records = (uint64_t*)hp;
+    return GA_OK;
+#else
+    (void)host_records;
+    return GA_EINVAL;
+#endif
 }
 
 ga_status ga_bsem_bench(ga_stream_t stream, const ga_bsem_cfg* cfg, uint64_t* sems, uint64_t* out) {

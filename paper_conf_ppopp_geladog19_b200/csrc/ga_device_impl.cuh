@@ -57,6 +57,12 @@ constexpr int kMaxLevels = 48;
 #ifndef GA_TREE_SPIN_CAP
 #define GA_TREE_SPIN_CAP 256     // max __nanosleep backoff (ns) of a blocked TBuddy wait
 #endif
+#ifndef GA_WW_BINS
+#define GA_WW_BINS 1             // 1: bin claims of all class groups of a warp run together
+#endif
+#ifndef GA_WW_TREE
+#define GA_WW_TREE 1             // 1: TBuddy node claims of all order groups run together
+#endif
 #ifndef GA_OPT_LOAD_GATED
 #define GA_OPT_LOAD_GATED 0      // 1: optimistic (TBuddy) waits decide on a plain load first
 #endif
@@ -99,6 +105,32 @@ static __device__ __forceinline__ void red_add_release(uint64_t* p, uint64_t v) 
 static __device__ __forceinline__ void fence() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
 static __device__ __forceinline__ void fence_sc() { __threadfence(); }
 static __device__ __forceinline__ void stat_add(const ga_desc* h, int i, uint64_t v) { a_add(&h->stats[i], v); }
+
+// GA_DEBUG builds: a spin loop that runs ~2^20 times records (site, ids, a, b)
+// into host-mapped memory, readable while a kernel hangs (tools/hang_probe.py)
+#ifndef GA_DEBUG
+#define GA_DEBUG 0
+#endif
+#if GA_DEBUG
+static __device__ uint64_t* g_ga_dbg;
+#define SPIN_NOTE(cnt, site, a, b) spin_note((cnt), (site), (uint64_t)(a), (uint64_t)(b))
+#define GA_DBG_CNT uint32_t dbg_cnt = 0
+static __device__ __noinline__ void spin_note(uint32_t& cnt, int site, uint64_t a, uint64_t b) {
+    if ((++cnt & ((1u << 18) - 1)) != 0 || !g_ga_dbg) return;
+    uint64_t* dbg = g_ga_dbg;
+    unsigned long long i = atomicAdd((unsigned long long*)&dbg[0], 1ull);
+    if (i >= 255) return;
+    uint32_t w; asm volatile("mov.u32 %0, %%warpid;" : "=r"(w));
+    uint32_t sm; asm volatile("mov.u32 %0, %%smid;" : "=r"(sm));
+    uint32_t ln; asm volatile("mov.u32 %0, %%laneid;" : "=r"(ln));
+    volatile uint64_t* r = (volatile uint64_t*)&dbg[8 + i * 4];
+    r[0] = (uint64_t)site; r[1] = ((uint64_t)sm << 32) | (w << 8) | ln; r[2] = a; r[3] = b;
+    __threadfence_system();
+}
+#else
+#define SPIN_NOTE(cnt, site, a, b) ((void)0)
+#define GA_DBG_CNT ((void)0)
+#endif
 
 static __device__ __forceinline__ uint32_t hash32(uint32_t x) {
     x ^= x >> 16; x *= 0x7feb352dU; x ^= x >> 15; x *= 0x846ca68bU; x ^= x >> 16; return x;
@@ -186,6 +218,7 @@ static __device__ __forceinline__ bool bsem_trywait(uint64_t* s, uint32_t N, uin
 // Alg. 1 core (documentation at bsem_wait below).
 template <bool kExact, class Spin>
 static __device__ __noinline__ int bsem_wait_impl(uint64_t* s, uint32_t N, uint32_t B, Spin spin) {
+    GA_DBG_CNT;
     const uint64_t dn = (uint64_t)N << 32;
     uint64_t w;
     if (kExact) {
@@ -213,6 +246,7 @@ static __device__ __noinline__ int bsem_wait_impl(uint64_t* s, uint32_t N, uint3
                 w = ld_rlx(s);
                 if (!(sem_C(w) < (int32_t)N && (int64_t)sem_C(w) + sem_D(w) >= 0)) break;
                 spin();
+                SPIN_NOTE(dbg_cnt, 1, (uint64_t)(uintptr_t)s, w);
                 __nanosleep(ns);
                 if (ns < 2048) ns <<= 1;
             }
@@ -244,6 +278,7 @@ static __device__ __noinline__ int bsem_wait_impl(uint64_t* s, uint32_t N, uint3
         uint32_t ns = 32;
         while (sem_C(w) < (int32_t)N && (int64_t)sem_C(w) + sem_D(w) >= 0) {                    // R-2
             spin();
+            SPIN_NOTE(dbg_cnt, 2, (uint64_t)(uintptr_t)s, w);
             __nanosleep(ns);
             if (ns < GA_TREE_SPIN_CAP) ns <<= 1;
             w = ld_rlx(s);
@@ -269,6 +304,7 @@ static __device__ __noinline__ int bsem_wait_impl(uint64_t* s, uint32_t N, uint3
         uint32_t ns = 32;
         while (sem_C(w) < (int32_t)N && (int64_t)sem_C(w) + sem_D(w) >= 0) {                    // R-2
             spin();
+            SPIN_NOTE(dbg_cnt, 3, (uint64_t)(uintptr_t)s, w);
             __nanosleep(ns);
             if (ns < GA_TREE_SPIN_CAP) ns <<= 1;
             w = ld_rlx(s);
@@ -397,6 +433,7 @@ static __device__ __forceinline__ void tree_publish(const ga_desc* h, int n, uin
 // claim up to `need` available nodes of level n from one bitmap word (the
 // caller holds `need` units of tsem[n]); returns the claimed mask, word in *wj
 static __device__ __noinline__ uint64_t tree_claim_word(const ga_desc* h, int n, int need, uint32_t seed, uint64_t* wj) {
+    GA_DBG_CNT;
     HB3 b = level_hb(h, n);
     uint32_t ns = 32;
 #if GA_LVL_HINT
@@ -425,6 +462,7 @@ static __device__ __noinline__ uint64_t tree_claim_word(const ga_desc* h, int n,
             }
         }
         j = -1;
+        SPIN_NOTE(dbg_cnt, 4, ((uint64_t)n << 32) | (uint32_t)need, seed);
         __nanosleep(ns); if (ns < 1024) ns <<= 1;
         seed = hash32(seed + 1);
     }
@@ -455,6 +493,7 @@ static __device__ __noinline__ int64_t tree_alloc_one(const ga_desc* h, int o) {
 // (R-19); otherwise mark x available with ONE CAS on the word holding both
 // siblings (R-21), so two siblings never both end up available.
 static __device__ __noinline__ void tree_free(const ga_desc* h, int n, uint64_t x) {
+    GA_DBG_CNT;
     uint32_t ns = 32;
     for (;;) {
         HB3 b = level_hb(h, n);
@@ -472,6 +511,7 @@ static __device__ __noinline__ void tree_free(const ga_desc* h, int n, uint64_t 
                 }
                 bsem_signal(tsem_ptr(h, n), 1, 0);            // buddy claimed meanwhile: give back
             } else {
+                SPIN_NOTE(dbg_cnt, 5, ((uint64_t)n << 56) | x, w);
                 __nanosleep(ns); if (ns < 1024) ns <<= 1;     // the buddy's unit is held by a claimer
             }
             continue;
@@ -554,6 +594,7 @@ static __device__ __noinline__ int64_t chunk_acquire(const ga_desc* h, uint32_t 
 // Claim up to `need` free pages from ONE chunk of arena A (caller holds `need`
 // units of psem[A]): one atomicOr per attempt.  Returns the page mask, chunk in *ch_out.
 static __device__ __noinline__ uint64_t page_claim(const ga_desc* h, uint32_t A, int need, uint64_t* ch_out) {
+    GA_DBG_CNT;
     HB3 fb = arena_hb(h, A, kAhbFpc);
     uint32_t seed = scatter_seed();
     uint32_t ns = 32;
@@ -583,6 +624,7 @@ static __device__ __noinline__ uint64_t page_claim(const ga_desc* h, uint32_t A,
                 if (u == ~0ull) hb3_clear_summarised(fb, ch, &h->chunk_used[ch], ~0ull);
             }
         }
+        SPIN_NOTE(dbg_cnt, 6, A, need);
         __nanosleep(ns); if (ns < 1024) ns <<= 1;
         seed = hash32(seed + 5);
     }
@@ -668,6 +710,7 @@ static __device__ __noinline__ uint64_t bin_claim_page(const ga_desc* h, uint64_
 // the hint's chunk first, then the (A, c) summary.  Spins until one shows up
 // (the caller holds units, so a free slot exists or is being published).
 static __device__ __noinline__ uint64_t bin_find_chunk(const ga_desc* h, uint32_t A, int c, uint64_t* mask_out) {
+    GA_DBG_CNT;
     uint32_t hp = ld_rlx32(&h->hint[A * kNcls + c]);
     if (hp < h->pages) {
         uint64_t m = ld_rlx(nonfull_word(h, hp >> kChunkShift, c));
@@ -693,6 +736,7 @@ static __device__ __noinline__ uint64_t bin_find_chunk(const ga_desc* h, uint32_
                 hb3_clear_summarised(nb, ch, nonfull_word(h, ch, c), 0);    // stale summary bit
             }
         }
+        SPIN_NOTE(dbg_cnt, 7, ((uint64_t)A << 8) | c, ns);
         __nanosleep(ns); if (ns < 1024) ns <<= 1;
         seed = hash32(seed + 7);
     }
@@ -792,6 +836,7 @@ static __device__ __noinline__ void reclaim_all(const ga_desc* h) {
 // order semaphores can send a lane up the tree while another lane's split is
 // still in flight.  Retry while the tree shows supply; drain reclamation once.
 static __device__ __noinline__ int64_t tree_alloc_one_retry(const ga_desc* h, int o) {
+    GA_DBG_CNT;
     bool drained = false;
     uint32_t ns = 64;
     for (int attempt = 0; attempt < 32; attempt++) {
@@ -803,6 +848,7 @@ static __device__ __noinline__ int64_t tree_alloc_one_retry(const ga_desc* h, in
             drained = true;
             continue;
         }
+        SPIN_NOTE(dbg_cnt, 8, o, attempt);
         __nanosleep(ns); if (ns < 4096) ns <<= 1;
     }
     return -1;
@@ -992,6 +1038,7 @@ static __device__ __noinline__ int bin_grow_leader(const ga_desc* h, uint32_t A,
 // promised -- so no waiter depends on work behind a warp barrier.
 // Returns m (or -1 after retracting every E); *xpart = the partly used node.
 static __device__ __noinline__ int tree_climb_leader(const ga_desc* h, int o, uint32_t N, uint32_t* Nm_out, uint64_t* xpart) {
+    GA_DBG_CNT;
     int m = o;
     uint32_t Nm = N;
     uint32_t ns = 128;
@@ -1011,6 +1058,7 @@ static __device__ __noinline__ int tree_climb_leader(const ga_desc* h, int o, ui
         // No false resource starvation: while splits are in flight
         // (cold start) or units are visible at some order >= o, re-climb
         if (m >= 0 || attempt >= 8 || !tree_has_supply(h, o, attempt < 2)) break;
+        SPIN_NOTE(dbg_cnt, 9, o, attempt);
         __nanosleep(ns); if (ns < 8192) ns <<= 1;
     }
     *Nm_out = Nm;
@@ -1101,7 +1149,7 @@ static __device__ __noinline__ uint64_t ga_malloc_off(const ga_desc* h, uint64_t
         __syncwarp(bins);                                          // all production of this warp is done
         r = __shfl_sync(bins, r, leader);
         const unsigned acq = __ballot_sync(bins, r == kAcquired);
-        if (r == kAcquired) my = bin_claim_collective(h, acq, grp, A, key);
+        if (r == kAcquired) my = bin_claim_collective(h, GA_WW_BINS ? acq : grp, grp, A, key);
         else if (r == kRGrown) {
             // hand the new slots out: rank -> (run, page, slot), group-local
             nruns = __shfl_sync(grp, nruns, leader);
@@ -1135,7 +1183,7 @@ static __device__ __noinline__ uint64_t ga_malloc_off(const ga_desc* h, uint64_t
         Nm = __shfl_sync(trees, Nm, leader);
         xpart = __shfl_sync(trees, xpart, leader);
         const unsigned ok = __ballot_sync(trees, m >= 0);
-        if (m >= 0) my = tree_claim_collective(h, ok, grp, o, m, Nm, xpart);
+        if (m >= 0) my = tree_claim_collective(h, GA_WW_TREE ? ok : grp, grp, o, m, Nm, xpart);
         if (my == kNull) {
             int64_t x = tree_alloc_one_retry(h, o);
             if (x >= 0) {
