@@ -57,12 +57,6 @@ constexpr int kMaxLevels = 48;
 #ifndef GA_TREE_SPIN_CAP
 #define GA_TREE_SPIN_CAP 256     // max __nanosleep backoff (ns) of a blocked TBuddy wait
 #endif
-#ifndef GA_WW_BINS
-#define GA_WW_BINS 1             // 1: bin claims of all class groups of a warp run together
-#endif
-#ifndef GA_WW_TREE
-#define GA_WW_TREE 1             // 1: TBuddy node claims of all order groups run together
-#endif
 #ifndef GA_OPT_LOAD_GATED
 #define GA_OPT_LOAD_GATED 0      // 1: optimistic (TBuddy) waits decide on a plain load first
 #endif
@@ -932,178 +926,165 @@ static __device__ __noinline__ uint64_t bin_malloc_lane(const ga_desc* h, uint32
     return kNull;
 }
 
-// ---- warp-wide collective steps -------------------------------------------------
-// A warp's lanes are grouped by size class (one group per class, mask `grp`).
-// The collective steps below run for ALL groups of the warp at once: every
-// warp-sync intrinsic uses the mask of all participating lanes (`live`), each
-// lane reading from its own group's leader, and __syncwarp(live) reconverges
-// the warp before each atomic, so the groups' atomics issue in the same
-// instruction instead of one group after another.
-
-// ---- bins: one slot per lane; every group of `live` holds its units ------------
-// Lanes spread over the chunk's non-full pages by their rank in the group (each
-// thread walks the number of elements its index dictates); lanes
-// that picked the same page regroup, and that page gets ONE atomicOr for all of them.
-static __device__ __noinline__ uint64_t bin_claim_collective(const ga_desc* h, unsigned live, unsigned grp, uint32_t A, int c) {
+// ---- bins: collective claim of one slot per lane (units already acquired) ----
+// Lanes spread over the chunk's non-full pages by their rank (each thread walks
+// the number of elements its index dictates), lanes that picked
+// the same page regroup and that page gets ONE atomicOr for all of them.
+static __device__ __noinline__ uint64_t bin_claim_collective(const ga_desc* h, unsigned grp, uint32_t A, int c) {
     const uint32_t lane = lane_id();
     const uint32_t per_page = slots_of(c) < 64 ? slots_of(c) : 64;
     const uint64_t csz = 16ull << c;
     uint64_t my = kNull;
+    unsigned unsat = grp;                                   // lanes still without a slot (this lane included)
     for (;;) {
-        const unsigned mine = live & grp;                        // my group's lanes still without a slot
-        const int L = __ffs(mine) - 1;
+        const int L = __ffs(unsat) - 1;
         uint64_t ch = 0, m = 0;
         if ((int)lane == L) ch = bin_find_chunk(h, A, c, &m);
-        __syncwarp(live);
-        ch = __shfl_sync(live, ch, L);
-        m = __shfl_sync(live, m, L);
-        const uint32_t q = __popc(mine & lanemask_lt());
+        ch = __shfl_sync(unsat, ch, L);
+        m = __shfl_sync(unsat, m, L);
+        const uint32_t q = __popc(unsat & lanemask_lt());
         const uint32_t np = __popcll(m);
         const uint64_t page = ch * kChunkPages + nth_set(m, (q / per_page) % np);
-        const unsigned pg = __match_any_sync(live, (page << 3) | (uint64_t)c);
+        const unsigned pg = __match_any_sync(unsat, page);
         const int pl = __ffs(pg) - 1;
         uint64_t got = 0;
         int wi = 0;
         if ((int)lane == pl) got = bin_claim_page(h, page, A, c, __popc(pg), &wi);
-        __syncwarp(live);
-        got = __shfl_sync(live, got, pl);
-        wi = __shfl_sync(live, wi, pl);
+        got = __shfl_sync(pg, got, pl);
+        wi = __shfl_sync(pg, wi, pl);
         const uint32_t pr = __popc(pg & lanemask_lt());
         if (pr < (uint32_t)__popcll(got)) my = (page << kPageShift) + (uint64_t)(wi * 64 + nth_set(got, pr)) * csz;
-        live = __ballot_sync(live, my == kNull);
-        if (my != kNull) break;                                  // a served lane leaves
+        unsat = __ballot_sync(unsat, my == kNull);
+        if (my != kNull) break;                             // a satisfied lane leaves the group
     }
     return my;
 }
 
-// ---- bins: growth, done by the group's leader before any warp-wide sync ----------
-// (a leader blocked in a semaphore wait may be waiting for this very production
-// in another warp, so production must never wait on a warp barrier).  The leader
-// accounts ceil(N/slots) pages on the arena page semaphore, tracks them one chunk
-// at a time (one atomicOr claims several pages: the collective chunk-list split
-// of P:L1282-1292), initialises every new bin (the group keeps the first N
-// slots) and publishes the spare slots with one signal.  The pages are recorded
-// as (chunk, page mask) runs for the lanes.  Returns the number of runs, 0 on
-// failure (every E retracted).
-constexpr int kMaxRuns = 16;
-static __device__ __noinline__ int bin_grow_leader(const ga_desc* h, uint32_t A, int c, uint32_t N,
-                                                   uint64_t* run_ch, uint64_t* run_pm) {
-    const uint32_t slots = slots_of(c);
-    const uint32_t Bp = slots * ((N + slots - 1) / slots);                 // R-8
-    const uint32_t k = Bp / slots;
-    int nruns = 0;
-    uint32_t pages_left = k, left = N;
-    uint64_t last_page = 0;
-    if (bsem_wait(psem_ptr(h, A), k, kChunkPages, ArenaSpin{h, A}) == kGrow) {
-        reclaim_arena(h, A, -1, kReclaimKeep);                              // delegated work first
-        int64_t nc = chunk_acquire(h, A, k);
-        if (nc < 0) {
-            bsem_signal(psem_ptr(h, A), 0, kChunkPages - k);
-            bsem_signal(sem_ptr(h, A, c), 0, Bp - N);
-            return 0;
-        }
-        bsem_signal(psem_ptr(h, A), kChunkPages - k, kChunkPages - k);
-        run_ch[0] = (uint64_t)nc;
-        run_pm[0] = k >= 64 ? ~0ull : ((1ull << k) - 1);
-        nruns = 1;
-        pages_left = 0;
-    }
-    while (pages_left) {
-        uint64_t ch;
-        uint64_t pm = page_claim(h, A, (int)pages_left, &ch);
-        run_ch[nruns] = ch; run_pm[nruns] = pm; nruns++;
-        pages_left -= __popcll(pm);
-    }
-    for (int i = 0; i < nruns; i++) {
-        uint64_t pm = run_pm[i];
-        while (pm) {
-            uint64_t p = run_ch[i] * kChunkPages + (uint64_t)(__ffsll((long long)pm) - 1);
-            pm &= pm - 1;
-            bin_init(h, p, A, c, left < slots ? left : slots);
-            left -= left < slots ? left : slots;
-            last_page = p;
-        }
-    }
-    stat_add(h, kStatBinGrow, k);
-    st_rlx32(&h->hint[A * kNcls + c], (uint32_t)last_page);
-    bsem_signal(sem_ptr(h, A, c), Bp - N, Bp - N);                          // release the spare slots
-    return nruns;
-}
-
-// ---- TBuddy: the leader's climb (Alg. 1 per order) ------------------
-// One bulk wait of N units per order (batch 2, B' = 2*ceil(N/2)); on GROW the
-// group climbs with N_{k+1} = ceil(N_k / 2) until an order m grants N_m nodes.
-// If the last node is only partly used, the leader claims it first and
-// publishes its unused right parts right away -- the E each level's GROW
-// promised -- so no waiter depends on work behind a warp barrier.
-// Returns m (or -1 after retracting every E); *xpart = the partly used node.
-static __device__ __noinline__ int tree_climb_leader(const ga_desc* h, int o, uint32_t N, uint32_t* Nm_out, uint64_t* xpart) {
-    GA_DBG_CNT;
-    int m = o;
-    uint32_t Nm = N;
-    uint32_t ns = 128;
-    for (int attempt = 0;; attempt++) {
-        m = o; Nm = N;
-        for (;;) {
-            if (m > (int)h->L) {                                            // nothing to grow from: retract every E
-                uint32_t nk = N;
-                for (int k = o; k < m; k++) { bsem_signal(tsem_ptr(h, k), 0, 2 * ((nk + 1) >> 1) - nk); nk = (nk + 1) >> 1; }
-                m = -1;
-                break;
-            }
-            if (bsem_wait_fast(tsem_ptr(h, m), Nm, 2 * ((Nm + 1) >> 1), NoSpin()) == kAcquired) break;
-            Nm = (Nm + 1) >> 1;
-            m++;
-        }
-        // No false resource starvation: while splits are in flight
-        // (cold start) or units are visible at some order >= o, re-climb
-        if (m >= 0 || attempt >= 8 || !tree_has_supply(h, o, attempt < 2)) break;
-        SPIN_NOTE(dbg_cnt, 9, o, attempt);
-        __nanosleep(ns); if (ns < 8192) ns <<= 1;
-    }
-    *Nm_out = Nm;
-    *xpart = kNull;
-    const int s = m - o;
-    if (m >= 0 && s > 0 && (N & ((1u << s) - 1))) {
-        uint64_t wj;
-        uint64_t got = tree_claim_word(h, m, 1, scatter_seed(), &wj);
-        const uint64_t x = wj * 64 + (uint64_t)(__ffsll((long long)got) - 1);
-        const uint64_t keep = N & ((1u << s) - 1);                          // lanes served by x
-        for (int j = 0; j < s; j++) {
-            const uint64_t pj = (keep + (1ull << j) - 1) & ~((1ull << j) - 1);
-            if ((pj >> j) & 1) tree_publish(h, o + j, ((x << s) + pj) >> j, 1);
-        }
-        *xpart = x;
-    }
-    return m;
-}
-
-// ---- TBuddy: full nodes claimed for all groups of `live` at once ---------------
-// (only claims: the units are held, nothing is produced here)
-static __device__ __noinline__ uint64_t tree_claim_collective(const ga_desc* h, unsigned live, unsigned grp, int o, int m,
-                                                              uint32_t Nm, uint64_t xpart) {
+// ---- bins: collective growth (class semaphore said GROW for the group) ------
+// The leader accounts ceil(N/slots) pages on the arena page semaphore and
+// tracks them one chunk at a time (one atomicOr claims several pages: the
+// collective chunk-list split of P:L1282-1292); every lane computes its page
+// and slot, the first lane of each page initialises that bin, then the leader
+// publishes the spare slots with one signal.  Returns kNull for every lane if
+// the group could not grow (the caller degrades to per-lane waits).
+static __device__ __noinline__ uint64_t bin_grow_collective(const ga_desc* h, unsigned grp, uint32_t A, int c) {
     const uint32_t lane = lane_id();
     const int leader = __ffs(grp) - 1;
     const uint32_t N = __popc(grp), rank = __popc(grp & lanemask_lt());
-    const int s = m - o;
-    const uint32_t nfull = xpart == kNull ? Nm : Nm - 1;                   // nodes serving 2^s lanes each
-    const uint32_t full_lanes = nfull << s;
+    const uint32_t slots = slots_of(c);
+    const uint32_t Bp = slots * ((N + slots - 1) / slots);                 // R-8
+    const uint32_t k = Bp / slots;
+    const uint64_t csz = 16ull << c;
     uint64_t my = kNull;
-    if (rank >= full_lanes) {                                              // lanes of the partly used node
-        const uint64_t pg = ((xpart << s) + (rank - full_lanes)) << o;
-        st_rlx32(&h->kind[pg], kKindTree | (uint32_t)o);
-        my = pg << kPageShift;
+    int mode = 0;                                                            // 0 claim pages, 1 fresh chunk, -1 fail
+    uint64_t ch = 0, pm = 0;
+    if ((int)lane == leader) {
+        if (bsem_wait(psem_ptr(h, A), k, kChunkPages, ArenaSpin{h, A}) == kGrow) {
+            reclaim_arena(h, A, -1, kReclaimKeep);                           // delegated work first
+            int64_t nc = chunk_acquire(h, A, k);
+            if (nc < 0) {
+                bsem_signal(psem_ptr(h, A), 0, kChunkPages - k);
+                bsem_signal(sem_ptr(h, A, c), 0, Bp - N);
+                mode = -1;
+            } else {
+                bsem_signal(psem_ptr(h, A), kChunkPages - k, kChunkPages - k);
+                mode = 1; ch = (uint64_t)nc; pm = k >= 64 ? ~0ull : ((1ull << k) - 1);
+            }
+        }
     }
-    live = __ballot_sync(live, nfull > 0);
-    if (nfull == 0) return my;
-    uint32_t served = 0;                                                   // lanes served from full nodes
-    const uint32_t seed = scatter_seed();
-    for (;;) {
+    mode = __shfl_sync(grp, mode, leader);
+    if (mode < 0) return kNull;
+    uint32_t served = 0, pages_left = k;
+    uint64_t last_page = 0;
+    while (pages_left) {
+        if (mode == 0 && (int)lane == leader) pm = page_claim(h, A, (int)pages_left, &ch);
+        ch = __shfl_sync(grp, ch, leader);
+        pm = __shfl_sync(grp, pm, leader);
+        const uint32_t np = __popcll(pm);
+        const uint32_t cap = np * slots;
+        if (rank >= served && rank < served + cap) {
+            const uint32_t r = rank - served;
+            const uint64_t p = ch * kChunkPages + nth_set(pm, r / slots);
+            my = (p << kPageShift) + (uint64_t)(r % slots) * csz;
+            if (r % slots == 0) {
+                const uint32_t left = N - served - (r / slots) * slots;
+                bin_init(h, p, A, c, left < slots ? left : slots);
+            }
+        }
+        last_page = ch * kChunkPages + nth_set(pm, np - 1);
+        served += cap < N - served ? cap : N - served;
+        pages_left -= np;
+        mode = 0;
+    }
+    __syncwarp(grp);
+    if ((int)lane == leader) {
+        stat_add(h, kStatBinGrow, k);
+        st_rlx32(&h->hint[A * kNcls + c], (uint32_t)last_page);
+        bsem_signal(sem_ptr(h, A, c), Bp - N, Bp - N);                      // release: bins are initialised
+    }
+    return my;
+}
+
+// ---- TBuddy, group path -------------------------------------------------------
+// One bulk wait of N units per order for the group (batch 2, B' = 2*ceil(N/2));
+// on GROW the group climbs with N_{k+1} = ceil(N_k / 2), claims N_m nodes at the
+// granting level m and splits them down: each claimed node serves 2^(m-o)
+// lanes, the unused right parts of the last node are published.  Returns kNull
+// for every lane if the tree could not serve the whole group.
+static __device__ __noinline__ uint64_t tree_malloc_group(const ga_desc* h, unsigned grp, int o) {
+    const uint32_t lane = lane_id();
+    const int leader = __ffs(grp) - 1;
+    const uint32_t N = __popc(grp), rank = __popc(grp & lanemask_lt());
+    int m = o;
+    uint32_t Nm = N;
+    if ((int)lane == leader) {
+        uint32_t ns = 128;
+        for (int attempt = 0;; attempt++) {
+            m = o; Nm = N;
+            for (;;) {
+                if (m > (int)h->L) {                         // nothing to grow from: retract every E
+                    uint32_t nk = N;
+                    for (int k = o; k < m; k++) { bsem_signal(tsem_ptr(h, k), 0, 2 * ((nk + 1) >> 1) - nk); nk = (nk + 1) >> 1; }
+                    m = -1;
+                    break;
+                }
+                if (bsem_wait_fast(tsem_ptr(h, m), Nm, 2 * ((Nm + 1) >> 1), NoSpin()) == kAcquired) break;
+                Nm = (Nm + 1) >> 1;
+                m++;
+            }
+            // No false resource starvation: while splits are in flight
+            // (cold start) or units are visible at some order >= o, re-climb
+            if (m >= 0 || attempt >= 8 || !tree_has_supply(h, o, attempt < 2)) break;
+            __nanosleep(ns); if (ns < 8192) ns <<= 1;
+        }
+    }
+    m = __shfl_sync(grp, m, leader);
+    if (m < 0) return kNull;
+    Nm = __shfl_sync(grp, Nm, leader);
+    const int s = m - o;
+    uint64_t my = kNull;
+    uint32_t served = 0;
+    uint32_t seed = scatter_seed();
+    while (served < N) {
         uint64_t wj = 0, got = 0;
-        if ((int)lane == leader) got = tree_claim_word(h, m, (int)(nfull - (served >> s)), seed, &wj);
-        __syncwarp(live);
-        wj = __shfl_sync(live, wj, leader);
-        got = __shfl_sync(live, got, leader);
+        if ((int)lane == leader) got = tree_claim_word(h, m, (int)(Nm - (served >> s)), seed, &wj);
+        wj = __shfl_sync(grp, wj, leader);
+        got = __shfl_sync(grp, got, leader);
+        {
+            const uint32_t nn = __popcll(got), rem = N - served;
+            if ((nn << s) >= rem && s > 0) {
+                // the last node is split: its unused right parts [pos, 2^s) decompose into
+                // one aligned block per set bit j of the running position (E at each level
+                // o + j); the group's lanes publish them in parallel, lane q doing level o + q
+                const uint64_t xlast = wj * 64 + (63 - __clzll((long long)got));
+                const uint64_t keep = rem - ((nn - 1) << s);
+                for (uint32_t j = rank; j < (uint32_t)s; j += N) {
+                    // running position before level j = keep rounded up to a multiple of 2^j
+                    const uint64_t pj = (keep + (1ull << j) - 1) & ~((1ull << j) - 1);
+                    if ((pj >> j) & 1) tree_publish(h, o + (int)j, ((xlast << s) + pj) >> j, 1);
+                }
+            }
+        }
         const uint32_t cap = (uint32_t)__popcll(got) << s;
         if (rank >= served && rank < served + cap) {
             const uint32_t r = rank - served;
@@ -1112,78 +1093,34 @@ static __device__ __noinline__ uint64_t tree_claim_collective(const ga_desc* h, 
             st_rlx32(&h->kind[pg], kKindTree | (uint32_t)o);
             my = pg << kPageShift;
         }
-        served += cap;
-        const bool done = served >= full_lanes;                              // uniform within the group
-        live = __ballot_sync(live, !done);
-        if (done) break;
+        served += cap < N - served ? cap : N - served;
     }
-    (void)N;
     return my;
 }
 
 // ---- the entry points ---------------------------------------------------------
-enum { kRGrown = 2, kRFailed = 3 };
 static __device__ __noinline__ uint64_t ga_malloc_off(const ga_desc* h, uint64_t n) {
     const unsigned act = __activemask();
     const int key = size_key(h, n);
     const unsigned grp = __match_any_sync(act, key);
-    const unsigned bins = __ballot_sync(act, key >= 0 && key < kNcls);
-    const unsigned trees = __ballot_sync(act, key >= kNcls);
     if (key < 0) return kNull;
-    const uint32_t lane = lane_id();
-    const int leader = __ffs(grp) - 1;
-    const uint32_t N = __popc(grp), rank = __popc(grp & lanemask_lt());
-    uint64_t my = kNull;
+    uint64_t my;
     if (key < kNcls) {
         const uint32_t A = arena_of(h);
-        const uint32_t slots = slots_of(key);
-        int r = 0, nruns = 0;
-        uint64_t run_ch[kMaxRuns], run_pm[kMaxRuns];
-        if ((int)lane == leader) {                                 // every group's leader at once
+        const uint32_t N = __popc(grp), slots = slots_of(key);
+        const int leader = __ffs(grp) - 1;
+        int r = 0;
+        if ((int)lane_id() == leader)
             r = bsem_wait(sem_ptr(h, A, key), N, slots * ((N + slots - 1) / slots), ArenaSpin{h, A});
-            if (r == kGrow) {
-                nruns = bin_grow_leader(h, A, key, N, run_ch, run_pm);
-                r = nruns ? kRGrown : kRFailed;
-            }
-        }
-        __syncwarp(bins);                                          // all production of this warp is done
-        r = __shfl_sync(bins, r, leader);
-        const unsigned acq = __ballot_sync(bins, r == kAcquired);
-        if (r == kAcquired) my = bin_claim_collective(h, GA_WW_BINS ? acq : grp, grp, A, key);
-        else if (r == kRGrown) {
-            // hand the new slots out: rank -> (run, page, slot), group-local
-            nruns = __shfl_sync(grp, nruns, leader);
-            uint32_t base = 0;
-            const uint64_t csz = 16ull << key;
-            for (int i = 0; i < nruns; i++) {
-                uint64_t ch = 0, pm = 0;
-                if ((int)lane == leader) { ch = run_ch[i]; pm = run_pm[i]; }
-                ch = __shfl_sync(grp, ch, leader);
-                pm = __shfl_sync(grp, pm, leader);
-                const uint32_t cap = (uint32_t)__popcll(pm) * slots;
-                if (rank >= base && rank < base + cap) {
-                    const uint32_t q = rank - base;
-                    my = ((ch * kChunkPages + nth_set(pm, q / slots)) << kPageShift) + (uint64_t)(q % slots) * csz;
-                }
-                base += cap;
-            }
-        }
-        if (my == kNull) {                                         // R-27: the group degrades to per-lane waits
-            if ((int)lane == leader) stat_add(h, kStatFallback, 1);
-            my = bin_malloc_lane(h, A, key);
+        r = __shfl_sync(grp, r, leader);
+        my = r == kAcquired ? bin_claim_collective(h, grp, A, key) : bin_grow_collective(h, grp, A, key);
+        if (__any_sync(grp, my == kNull)) {                 // R-27: degrade to per-lane waits
+            if ((int)lane_id() == leader) stat_add(h, kStatFallback, 1);
+            if (my == kNull) my = bin_malloc_lane(h, A, key);
         }
     } else {
         const int o = key - kNcls;
-        int m = -1;
-        uint32_t Nm = 0;
-        uint64_t xpart = kNull;
-        if ((int)lane == leader) m = tree_climb_leader(h, o, N, &Nm, &xpart);
-        __syncwarp(trees);                                         // every split of this warp is published
-        m = __shfl_sync(trees, m, leader);
-        Nm = __shfl_sync(trees, Nm, leader);
-        xpart = __shfl_sync(trees, xpart, leader);
-        const unsigned ok = __ballot_sync(trees, m >= 0);
-        if (m >= 0) my = tree_claim_collective(h, GA_WW_TREE ? ok : grp, grp, o, m, Nm, xpart);
+        my = tree_malloc_group(h, grp, o);
         if (my == kNull) {
             int64_t x = tree_alloc_one_retry(h, o);
             if (x >= 0) {
@@ -1210,7 +1147,7 @@ static __device__ __noinline__ void ga_free_off(const ga_desc* h, uint64_t off) 
     const unsigned bins = __ballot_sync(act, is_bin);
     const unsigned trees = __ballot_sync(act, is_tree);
     if (is_tree) {
-        int n = (int)(k & 0xFF);                                   // order from the page kind (R-18)
+        int n = (int)(k & 0xFF);                               // order from the page kind (R-18)
         uint64_t x = p >> n;
         st_rlx32(&h->kind[p], 0);
         fence();
@@ -1239,13 +1176,12 @@ static __device__ __noinline__ void ga_free_off(const ga_desc* h, uint64_t off) 
     const unsigned g1 = __match_any_sync(bins, (p << 2) | (uint64_t)w);
     const uint64_t bit = 1ull << (slot & 63);
     const uint64_t mask = ((uint64_t)__reduce_or_sync(g1, (uint32_t)(bit >> 32)) << 32) | __reduce_or_sync(g1, (uint32_t)bit);
-    __syncwarp(bins);
-    if ((int)lane_id() == __ffs(g1) - 1) {                         // every word's leader at once
+    if ((int)lane_id() == __ffs(g1) - 1) {
         uint64_t* bw = page_bits(h, p);
         const uint64_t old = a_and(&bw[w], ~mask);
         const uint64_t v = valid_mask(c, w);
-        if ((old | ~v) == ~0ull) nonfull_set(h, p, c, A);         // the word was full: bin back in the list
-        if (((old & ~mask) & v) == 0) {                            // this word is empty: is the bin?
+        if ((old | ~v) == ~0ull) nonfull_set(h, p, c, A);     // the word was full: bin back in the list
+        if (((old & ~mask) & v) == 0) {                        // this word is empty: is the bin?
             uint64_t ww[4];
             ld_bitmap(bw, ww);
             bool empty = true;

@@ -5,7 +5,8 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import oracle, tracegen
 from paper_conf_ppopp_geladog19_b200.runner import GpuHeap, run_correctness
 torch.cuda.set_device(0)
-t = tracegen.d4_small(T=8192, R=8, heap_bytes=256 << 20)
+kmin = int(sys.argv[1]) if len(sys.argv) > 1 else 3
+t = tracegen.Trace("x", tracegen.mixed_sizes(tracegen.BASE_SEED + 40, 3, 8192, kmin, 15), 1, 256 << 20, 0)
 heap = GpuHeap(t.heap_bytes)
 run = run_correctness(heap, t.sizes, t.D)
 err, cs = oracle.check_log(run.log, t.R, t.T, t.D, t.heap_bytes)
@@ -27,6 +28,11 @@ for r in range(t.R):
     if bad:
         print("round", r, "overlaps:", len(bad))
         for a, b in bad[:6]:
-            print("  tid", a[2], "size", a[3], "off", hex(a[0]), "| tid", b[2], "size", b[3], "off", hex(b[0]),
-                  "| warps", a[2] // 32, b[2] // 32)
+            print("  tid", a[2], "size", a[3], "cls", cls(a[3]), "pages", hex(a[0] >> 12), hex(a[1] >> 12), "| tid", b[2], "size", b[3],
+                  "cls", cls(b[3]), "pages", hex(b[0] >> 12), hex(b[1] >> 12), "| warp/lane", a[2] // 32, a[2] % 32, b[2] // 32, b[2] % 32)
+            # same-class group mates of a in its warp
+            w = a[2] // 32
+            mates = [(tt % 32, int(log[2 * (r * T + tt)]['off']) >> 12, cls(int(log[2 * (r * T + tt)]['size'])))
+                     for tt in range(w * 32, w * 32 + 32) if cls(int(log[2 * (r * T + tt)]['size'])) == cls(a[3])]
+            print("     warp", w, "group (lane, page, cls):", mates)
         break
