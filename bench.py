@@ -186,6 +186,36 @@ def d3_sweep(ga, heap, stream, dev, T, args, sizes=(16, 32, 64, 128, 256, 512, 1
     return res
 
 
+def d2_bsem(ga, stream, dev, grid=148 * 8, block=256, iters=32):
+    """wait(k)/signal(k) per thread per iteration on a full grid; ops = wait+signal pairs."""
+    import torch
+    names = {0: "warp_aggregated_bulk", 1: "per_thread_bulk", 2: "per_thread_counting", 3: "plain_atomics"}
+    res = {}
+    sems = torch.zeros(148 * 4 + 8, dtype=torch.int64, device=dev)
+    out = torch.zeros(8, dtype=torch.int64, device=dev)
+    for n_sems in (1, 148):
+        for k in (1, 32, 0):
+            for v in (0, 1, 2, 3):
+                if v == 2 and k != 1:
+                    continue
+                cfg = ga.BsemCfg(variant=v, k=k, B=512, n_sems=n_sems, iters=iters, acquire_only=0, grid=grid,
+                                 block=block, seed=tracegen.BASE_SEED + 2)
+                best = None
+                for rep in range(3):
+                    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    e0.record(stream)
+                    ga.ga_bsem_bench(stream.cuda_stream, cfg, sems.data_ptr(), out.data_ptr())
+                    e1.record(stream)
+                    e1.synchronize()
+                    t = e0.elapsed_time(e1) / 1e3
+                    best = t if best is None else min(best, t)
+                o = out.cpu().numpy()
+                res[f"{names[v]}/k={k or 'rand'}/sems={n_sems}"] = {
+                    "pairs_per_s": grid * block * iters / best, "units_per_s": float(o[0]) / best,
+                    "quiescent_C_equals_produced": bool(o[4] == o[3]), "max_abs_D": int(o[5])}
+    return res
+
+
 # ----------------------------------------------------------------------------- our arm
 def main():
     ap = argparse.ArgumentParser()
@@ -378,6 +408,9 @@ def main():
         # ---- d3: warp-uniform sizes 16 B - 8 KiB (BASELINE configs[2]), malloc+free per
         # thread and round (D = 0), full grid; CUDA malloc on a bounded prefix of rounds
         out["d3_sweep"] = d3_sweep(ga, heap, stream, dev, T, args)
+
+        # ---- d2: bulk-semaphore microbenchmark (BASELINE configs[1], Sec. 5.1)
+        out["d2_bsem"] = d2_bsem(ga, stream, dev)
 
     print(json.dumps(out), flush=True)
     if dist:

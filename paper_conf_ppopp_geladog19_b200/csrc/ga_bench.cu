@@ -265,16 +265,12 @@ __global__ void k_bsem(ga_bsem_cfg cfg, uint64_t* sems, uint64_t* out, uint32_t 
             if (!cfg.acquire_only) atomicAdd(c, (unsigned long long)k + (tid & zero));
         }
     }
-    unsigned act = __activemask();
-    uint64_t g = granted, w = waits, b = batches, p = produced;
-    for (int o = 16; o; o >>= 1) {
-        g += __shfl_down_sync(act, g, o); w += __shfl_down_sync(act, w, o);
-        b += __shfl_down_sync(act, b, o); p += __shfl_down_sync(act, p, o);
-    }
-    if ((threadIdx.x & 31) == 0) {
-        atomicAdd((unsigned long long*)&out[0], g); atomicAdd((unsigned long long*)&out[1], w);
-        atomicAdd((unsigned long long*)&out[2], b); atomicAdd((unsigned long long*)&out[3], p);
-    }
+    // lanes leave their spin loops at different times: no converged-warp
+    // reduction here, plain per-thread atomics (ptxas aggregates uniform ones)
+    if (granted) atomicAdd((unsigned long long*)&out[0], (unsigned long long)granted);
+    if (waits) atomicAdd((unsigned long long*)&out[1], (unsigned long long)waits);
+    if (batches) atomicAdd((unsigned long long*)&out[2], (unsigned long long)batches);
+    if (produced) atomicAdd((unsigned long long*)&out[3], (unsigned long long)produced);
 }
 __global__ void k_bsem_final(uint32_t n_sems, const uint64_t* sems, uint64_t* out, uint32_t variant) {
     if (threadIdx.x || blockIdx.x) return;

@@ -1,0 +1,153 @@
+"""GPU checks at BASELINE sizes and of the microbenchmarks, through the C ABI.
+
+* config d4 at full occupancy (303,104 threads) in correctness mode: the whole
+  allocation log passes the oracle's checker, counts equal the oracle's (the
+  fit level: demand <= capacity, every call succeeds), the heap returns to the
+  empty snapshot after quiesce;
+* config d3 at full occupancy for a bin class and a TBuddy class;
+* the timed kernel (the launch configuration bench.py times) on the full d4
+  trace: counts equal the oracle's, heap empty after quiesce;
+* config d2, the bulk-semaphore microbenchmark: at quiescence D = 0 and C
+  equals the units produced minus the units still held; in acquire-only mode
+  (Fig. 5) per-thread bulk waits produce exactly ceil(demand/B)
+  batches (no over-production, P-2);
+* the L2-atomic peak microbenchmark runs and reports plausible rates.
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import tracegen
+from oracle import snapshot as S
+
+pytestmark = pytest.mark.gpu
+
+ga = pytest.importorskip("paper_conf_ppopp_geladog19_b200")
+from paper_conf_ppopp_geladog19_b200.runner import GpuHeap, run_correctness, run_timed  # noqa: E402
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _cuda():
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    torch.cuda.set_device(0)
+
+
+def _empty(heap):
+    heap.quiesce()
+    snap = heap.snapshot()
+    assert not S.check(S.parse(snap), require_reclaimed=True)
+    assert snap == oracle.snapshot_of_fresh(heap.heap_bytes)
+
+
+def test_d4_full_grid_correctness_fit():
+    """303,104 threads x 4 rounds of mixed 16 B - 64 KiB churn, 16 GiB heap (fit)."""
+    t = tracegen.d4_mixed("fit", R=4)
+    ref = oracle.run_trace(t.sizes, t.heap_bytes, t.D)
+    heap = GpuHeap(t.heap_bytes)
+    run = run_correctness(heap, t.sizes, t.D)
+    err, cs = oracle.check_log(run.log, t.R, t.T, t.D, t.heap_bytes)
+    assert err == 0, (err, cs)
+    assert run.counts["tag_errors"] == 0
+    assert run.counts["n_fail"] == ref.stats["n_malloc_fail"] == 0
+    assert run.counts["n_malloc"] == ref.stats["n_malloc"] and run.counts["n_free"] == ref.stats["n_free"]
+    _empty(heap)
+
+
+def test_d4_full_grid_pressure_valid():
+    """The bench workload (4 GiB, ~71 % live after rounding) in correctness mode."""
+    t = tracegen.d4_mixed("pressure", R=4)
+    heap = GpuHeap(t.heap_bytes)
+    run = run_correctness(heap, t.sizes, t.D)
+    err, cs = oracle.check_log(run.log, t.R, t.T, t.D, t.heap_bytes)
+    assert err == 0, (err, cs)
+    assert run.counts["tag_errors"] == 0
+    _empty(heap)
+
+
+@pytest.mark.parametrize("size", [16, 2048, 8192])
+def test_d3_full_grid_correctness(size):
+    t = tracegen.d3_uniform(size, R=2)
+    heap = GpuHeap(t.heap_bytes)
+    run = run_correctness(heap, t.sizes, t.D)
+    err, cs = oracle.check_log(run.log, t.R, t.T, t.D, t.heap_bytes)
+    assert err == 0, (err, cs)
+    assert run.counts["n_fail"] == 0 and run.counts["tag_errors"] == 0
+    _empty(heap)
+
+
+def test_timed_kernel_full_d4_counts():
+    """The kernel bench.py times, on the full bench trace: counts and empty heap."""
+    t = tracegen.d4_mixed("pressure")
+    ref = oracle.run_trace(t.sizes, t.heap_bytes, t.D, want_ok=False)
+    heap = GpuHeap(t.heap_bytes)
+    d = torch.from_numpy(t.sizes.view(np.int32)).cuda()
+    c = torch.zeros(8, dtype=torch.int64, device="cuda")
+    run_timed(heap, d, t.R, t.T, t.D, c)
+    torch.cuda.synchronize()
+    cc = c.cpu().numpy()
+    assert cc[0] == ref.stats["n_malloc"] and cc[1] == ref.stats["n_malloc_fail"] == 0
+    assert cc[2] == ref.stats["n_free"]
+    _empty(heap)
+
+
+def _bsem(variant, k, B, n_sems, iters, acquire_only, grid=148 * 4, block=256):
+    cfg = ga.BsemCfg(variant=variant, k=k, B=B, n_sems=n_sems, iters=iters, acquire_only=acquire_only,
+                     grid=grid, block=block, seed=tracegen.BASE_SEED + 2)
+    sems = torch.zeros(n_sems * 4 + 8, dtype=torch.int64, device="cuda")
+    out = torch.zeros(8, dtype=torch.int64, device="cuda")
+    ga.ga_bsem_bench(torch.cuda.current_stream().cuda_stream, cfg, sems.data_ptr(), out.data_ptr())
+    torch.cuda.synchronize()
+    o = out.cpu().numpy()
+    return {"granted": int(o[0]), "waits": int(o[1]), "batches": int(o[2]), "produced": int(o[3]),
+            "C": int(o[4]), "absD": int(o[5])}
+
+
+@pytest.mark.parametrize("variant", [0, 1])
+@pytest.mark.parametrize("k", [1, 4, 32, 0])
+@pytest.mark.parametrize("n_sems", [1, 148])
+def test_bsem_release_mode_invariants(variant, k, n_sems):
+    """wait(k) ... signal(k): at quiescence D = 0 and C = every unit produced."""
+    r = _bsem(variant, k, 512, n_sems, 8, 0)
+    assert r["absD"] == 0
+    assert r["C"] == r["produced"]
+    if k:
+        assert r["granted"] == 148 * 4 * 256 * 8 * k
+    assert r["batches"] * 512 == r["produced"]
+
+
+@pytest.mark.parametrize("B", [32, 512])
+def test_bsem_acquire_only_no_overproduction(B):
+    """Fig. 5 mode, per-thread waits of one unit: batches == ceil(demand / B) and
+    C = batches*B - demand (P-2 at GPU scale)."""
+    r = _bsem(1, 1, B, 1, 4, 1)
+    demand = 148 * 4 * 256 * 4
+    assert r["granted"] == demand
+    assert r["batches"] == -(-demand // B)
+    assert r["C"] == r["batches"] * B - demand and r["absD"] == 0
+
+
+def test_counting_and_plain_variants_run():
+    r = _bsem(2, 1, 512, 1, 4, 1)
+    assert r["granted"] == 148 * 4 * 256 * 4 and r["C"] >= 0
+    r = _bsem(3, 8, 512, 148, 4, 0)
+    assert r["C"] == 0
+
+
+def test_l2_atomic_bench_plausible():
+    buf = torch.zeros(148 * 8 * 256 * 4 + 8192, dtype=torch.int64, device="cuda")
+    sink = torch.zeros(8, dtype=torch.int64, device="cuda")
+    s = torch.cuda.current_stream()
+    rates = {}
+    for pat in range(6):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        iters = 16 if pat < 4 else 4
+        e0.record(s)
+        ga.ga_l2_atomic_bench(s.cuda_stream, pat, buf.data_ptr(), buf.numel(), iters, 148 * 8, 256, sink.data_ptr())
+        e1.record(s)
+        e1.synchronize()
+        rates[pat] = 148 * 8 * 256 * iters / (e0.elapsed_time(e1) / 1e3)
+    assert rates[1] > 1e10 and rates[0] > 1e10         # distinct-word atomics: > 10 Gatom/s
+    assert rates[2] < rates[0]                          # one hot word is slower than spread words
+    assert int(buf[0].item()) > 0
