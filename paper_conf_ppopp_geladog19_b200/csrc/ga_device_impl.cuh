@@ -98,6 +98,21 @@ static __device__ __forceinline__ void red_add_release(uint64_t* p, uint64_t v) 
 // fence_sc(): store -> load ordering for the clear-then-recheck (Dekker) patterns
 static __device__ __forceinline__ void fence() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
 static __device__ __forceinline__ void fence_sc() { __threadfence(); }
+// The re-check read of a clear-then-recheck (Dekker) pattern.  GA_RECHECK_RMW=1
+// reads the word with an atomicOr(0): RMWs on one address are totally ordered at
+// L2, and the read is issued only after the clearing RMW returned, so no SC fence
+// is needed; 0 uses fence.sc + a relaxed load.
+#ifndef GA_RECHECK_RMW
+#define GA_RECHECK_RMW 1
+#endif
+static __device__ __forceinline__ uint64_t recheck_read(uint64_t* p) {
+#if GA_RECHECK_RMW
+    return atomicOr((unsigned long long*)p, 0ull);
+#else
+    fence_sc();
+    return ld_rlx(p);
+#endif
+}
 static __device__ __forceinline__ void stat_add(const ga_desc* h, int i, uint64_t v) { a_add(&h->stats[i], v); }
 
 // GA_DEBUG builds: a spin loop that runs ~2^20 times records (site, ids, a, b)
@@ -139,10 +154,12 @@ static __device__ __forceinline__ uint64_t rotr(uint64_t x, uint32_t r) { r &= 6
 // index of the first set bit of x at or after position r (cyclic); x != 0
 static __device__ __forceinline__ uint32_t first_from(uint64_t x, uint32_t r) { return (uint32_t)((__ffsll((long long)rotr(x, r)) - 1 + r) & 63); }
 // mask of the lowest k set bits of x
+static __device__ __forceinline__ uint32_t nth_set(uint64_t x, uint32_t n);
 static __device__ __forceinline__ uint64_t lowest_bits(uint64_t x, int k) {
-    uint64_t m = 0;
-    while (k-- > 0 && x) { uint64_t b = x & (~x + 1); m |= b; x ^= b; }
-    return m;
+    if (k <= 0) return 0;
+    if (__popcll(x) <= k) return x;
+    const uint32_t pos = nth_set(x, (uint32_t)k - 1);       // the k-th set bit: keep bits <= pos
+    return x & (pos == 63 ? ~0ull : ((2ull << pos) - 1));
 }
 // position of the n-th (0-based) set bit of x
 // (branch-free popc binary search; __fns is emulated with a loop on sm_100a)
@@ -352,23 +369,20 @@ static __device__ __noinline__ void hb3_up_clear(HB3 b, uint32_t j) {
     uint64_t* w1 = hb3_w1(b);
     uint64_t bit = 1ull << (j & 63);
     uint64_t old = a_and(&w1[j >> 6], ~bit);
-    fence_sc();
-    if (ld_rlx(&b.w0[j]) != 0) { if (a_or(&w1[j >> 6], bit) == 0) a_or(&hb3_w2(b)[j >> 12], 1ull << ((j >> 6) & 63)); return; }
+    if (recheck_read(&b.w0[j]) != 0) { if (a_or(&w1[j >> 6], bit) == 0) a_or(&hb3_w2(b)[j >> 12], 1ull << ((j >> 6) & 63)); return; }
     if ((old & ~bit) != 0) return;
     uint32_t j1 = j >> 6;
     uint64_t* w2 = hb3_w2(b);
     uint64_t bit2 = 1ull << (j1 & 63);
     a_and(&w2[j1 >> 6], ~bit2);
-    fence_sc();
-    if (ld_rlx(&w1[j1]) != 0) a_or(&w2[j1 >> 6], bit2);
+    if (recheck_read(&w1[j1]) != 0) a_or(&w2[j1 >> 6], bit2);
 }
 // Bit i of w0 summarises an outside data word (*data).  Clear the bit when the
 // data says "empty", re-checking the data after the clear.
 static __device__ __noinline__ void hb3_clear_summarised(HB3 b, uint64_t i, const uint64_t* data, uint64_t empty_value) {
     uint64_t bit = 1ull << (i & 63);
     uint64_t old = a_and(&b.w0[i >> 6], ~bit);
-    fence_sc();
-    if (ld_rlx(data) != empty_value) { if (a_or(&b.w0[i >> 6], bit) == 0) hb3_up_set(b, (uint32_t)(i >> 6)); return; }
+    if (recheck_read((uint64_t*)data) != empty_value) { if (a_or(&b.w0[i >> 6], bit) == 0) hb3_up_set(b, (uint32_t)(i >> 6)); return; }
     if (old == bit) hb3_up_clear(b, (uint32_t)(i >> 6));
 }
 // a w0 word that looks non-zero, searched from a scattered start; -1 if none
@@ -561,9 +575,13 @@ static __device__ __noinline__ void nonfull_clear_if_full(const ga_desc* h, uint
     uint64_t* nf = nonfull_word(h, ch, c);
     uint64_t bit = 1ull << (p & (kChunkPages - 1));
     uint64_t old = a_and(nf, ~bit);
-    fence_sc();
     uint64_t w[4];
+#if GA_RECHECK_RMW
+    for (int i = 0; i < 4; i++) w[i] = i < words_of(c) ? recheck_read(&page_bits(h, p)[i]) : ~0ull;
+#else
+    fence_sc();
     ld_bitmap(page_bits(h, p), w);
+#endif
     if (ld_rlx32(&h->kind[p]) == kind_bin(A, c) && !page_full(w, c)) {
         if (a_or(nf, bit) == 0) hb3_set(arena_hb(h, A, kAhbNfc + c), ch);
         return;
