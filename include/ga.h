@@ -41,6 +41,9 @@ typedef struct {
     uint32_t bin_max;       /* 2048: largest bin class; >= 4096 goes to TBuddy (R-12)  */
     uint32_t n_classes;     /* 8 bin classes 16..2048                                  */
     uint32_t bitmap_bits;   /* 256: out-of-band bitmap bits per page                   */
+    uint32_t n_span_classes;/* 5 span classes 4..64 KiB, one 64-page chunk per span
+                               (DESIGN.md "Spans"); 0 in a GA_NSPAN=0 build          */
+    uint32_t span_max;      /* 65536: largest span class; larger sizes go to TBuddy    */
 } ga_layout_t;
 
 /* Device-resident heap descriptor (lives at the start of the metadata
@@ -57,14 +60,14 @@ typedef struct ga_desc {
     uint32_t* kind;           /* [pages] page kind (R-18)                               */
     uint64_t* chunk_used;     /* [nchunks] used pages; all ones when not owned          */
     uint32_t* chunk_owner;    /* [nchunks] arena + 1, 0 = in the tree                   */
-    uint64_t* chunk_nonfull;  /* [nchunks][8] per class: bins with a free slot          */
+    uint64_t* chunk_nonfull;  /* [nchunks][13] per class: bins / the span with a free slot */
     uint64_t* chunk_cand;     /* [nchunks] bins that went empty (reclaim candidates)    */
-    uint64_t* sem;            /* [n_arenas][8] class bulk semaphores, 32 B apart        */
+    uint64_t* sem;            /* [n_arenas][13] class bulk semaphores (8 bin + 5 span classes), 32 B apart */
     uint64_t* psem;           /* [n_arenas] page bulk semaphores, 32 B apart            */
-    uint32_t* hint;           /* [n_arenas][8] current bin page per class               */
-    uint64_t* ahb;            /* [n_arenas][10] chunk summaries (3-level bitsets): chunks
+    uint32_t* hint;           /* [n_arenas][13] current bin / span head page per class  */
+    uint64_t* ahb;            /* [n_arenas][2+13] chunk summaries (3-level bitsets): chunks
                                  with free pages, with reclaim candidates, with non-full
-                                 bins of class c (c = 0..7)                             */
+                                 bins (spans) of class c (c = 0..12)                    */
     uint64_t* avail;          /* TBuddy availability bitmaps, all levels (3-level each)  */
     uint64_t* tsem;           /* [L+1] per-order bulk semaphores, 32 B apart            */
     uint64_t* stats;          /* device counters, see ga_stats_t                        */
@@ -136,14 +139,20 @@ const char* ga_status_str(ga_status s);
  * Canonical snapshot (logical, little endian; the oracle writes the same format
  * independently, oracle/ga_oracle.c ora_snapshot):
  *   u64 magic "GASNAP01"; u64 heap_bytes; u64 pages; u64 page | (L+1) << 32;
- *   u64 min_class | n_classes << 32 | chunk_pages << 48;
+ *   u64 min_class | n_classes << 32 | n_span_classes << 40 | chunk_pages << 48;
  *   u8 kind[pages]: 0x00 free page inside an Available tree node (not its head),
  *                   0x40|n head of an Available node of order n, 0x80|n head of an
  *                   allocated user block of order n, 0x01 tail page of such a block,
- *                   0x02 free page of an arena chunk, 0x10|c bin of class c;
- *   for each bin page in ascending order: slots(c) bits, LSB first, padded to bytes;
+ *                   0x02 free page of an arena chunk, 0x10|c bin of class c,
+ *                   0x20|s first page of a span of span class s (blocks of page << s),
+ *                   0x04 any other page of a span;
+ *   for each bin or span head page in ascending order: its slots bits (a bin of
+ *                   class c: page / (min_class << c); a span of class s:
+ *                   chunk_pages >> s), LSB first, padded to bytes;
  *   for each level n = 0..L: 2^(L-n) availability bits, LSB first, padded to bytes;
- *   for each class: i64 sum over arenas of C, i64 max over arenas of |E-R|;
+ *   for each bin class, then each span class: i64 sum over arenas of C, i64 max
+ *                   over arenas of |E-R| (the oracle routes span sizes to TBuddy,
+ *                   as the paper does, and writes zeros for the span classes);
  *   i64 sum of page-semaphore C, i64 max |E-R|;
  *   for each order n = 0..L: i64 C, i64 E-R;
  *   u64 pending reclamation candidates.

@@ -29,7 +29,9 @@ K_FREE_INTERIOR = 0x00
 K_TREE_TAIL = 0x01
 K_CHUNK_FREE = 0x02
 K_CHUNK_HDR = 0x03
+K_SPAN_TAIL = 0x04
 K_BIN = 0x10      # | class index
+K_SPAN = 0x20     # | span class index (first page of a span)
 K_AVAIL = 0x40    # | order
 K_ALLOC = 0x80    # | order
 
@@ -42,11 +44,12 @@ class Snapshot:
     levels: int
     min_class: int
     ncls: int
+    nspan: int
     chunk_pages: int
     kind: np.ndarray              # u8[pages]
-    bins: dict                    # page -> np.ndarray(bool[slots])
+    bins: dict                    # page -> np.ndarray(bool[slots]) (bin pages and span heads)
     level_bits: list              # list of bool arrays, level n has 2^(L-n) entries
-    cls_C: np.ndarray             # i64[ncls]
+    cls_C: np.ndarray             # i64[ncls + nspan]: bin classes, then span classes
     cls_absD: np.ndarray
     page_C: int
     page_absD: int
@@ -55,7 +58,14 @@ class Snapshot:
     pending: int
 
     def slots(self, c: int) -> int:
-        return self.page // (self.min_class << c)
+        """Slots of class c (0..ncls-1 bins, ncls.. spans)."""
+        if c < self.ncls:
+            return self.page // (self.min_class << c)
+        return self.chunk_pages >> (c - self.ncls)
+
+    def page_class(self, p: int) -> int:
+        k = int(self.kind[p])
+        return (k & 0x0F) + (self.ncls if (k & 0xF0) == K_SPAN else 0)
 
     def reserved_pages(self) -> int:
         return self.pages - sum(int(b.sum()) << n for n, b in enumerate(self.level_bits))
@@ -83,13 +93,13 @@ def parse(buf: bytes) -> Snapshot:
     w = u64()
     page, levels = w & 0xFFFFFFFF, w >> 32
     w = u64()
-    min_class, ncls, chunk_pages = w & 0xFFFFFFFF, (w >> 32) & 0xFFFF, w >> 48
+    min_class, ncls, nspan, chunk_pages = w & 0xFFFFFFFF, (w >> 32) & 0xFF, (w >> 40) & 0xFF, w >> 48
     kind = b[pos:pos + pages].copy()
     pos += pages
     bins = {}
-    for p in np.nonzero((kind & 0xF0) == K_BIN)[0]:
+    for p in np.nonzero(((kind & 0xF0) == K_BIN) | ((kind & 0xF0) == K_SPAN))[0]:
         c = int(kind[p]) & 0x0F
-        s = page // (min_class << c)
+        s = page // (min_class << c) if (kind[p] & 0xF0) == K_BIN else chunk_pages >> c
         nb = (s + 7) // 8
         bits = np.unpackbits(b[pos:pos + nb], bitorder="little")[:s].astype(bool)
         bins[int(p)] = bits
@@ -101,13 +111,13 @@ def parse(buf: bytes) -> Snapshot:
         nb = (cnt + 7) // 8
         level_bits.append(np.unpackbits(b[pos:pos + nb], bitorder="little")[:cnt].astype(bool))
         pos += nb
-    cls = i64s(2 * ncls).reshape(ncls, 2)
+    cls = i64s(2 * (ncls + nspan)).reshape(ncls + nspan, 2)
     pg = i64s(2)
     tr = i64s(2 * levels).reshape(levels, 2)
     pending = u64()
     if pos != len(buf):
         raise ValueError(f"snapshot length mismatch: parsed {pos} of {len(buf)} bytes")
-    return Snapshot(heap_bytes, pages, page, levels, min_class, ncls, chunk_pages, kind, bins,
+    return Snapshot(heap_bytes, pages, page, levels, min_class, ncls, nspan, chunk_pages, kind, bins,
                     level_bits, cls[:, 0].copy(), cls[:, 1].copy(), int(pg[0]), int(pg[1]),
                     tr[:, 0].copy(), tr[:, 1].copy(), pending)
 
@@ -152,8 +162,16 @@ def check(s: Snapshot, require_reclaimed: bool = False) -> list:
             errs.append(f"tree block at page {p}: tail pages wrong")
     # chunks: aligned groups of chunk pages made only of free / bin / header pages
     cp = s.chunk_pages
-    chunkish = (s.kind == K_CHUNK_FREE) | ((s.kind & 0xF0) == K_BIN) | (s.kind == K_CHUNK_HDR)
+    chunkish = (s.kind == K_CHUNK_FREE) | ((s.kind & 0xF0) == K_BIN) | (s.kind == K_CHUNK_HDR) | \
+        (s.kind == K_SPAN_TAIL) | ((s.kind & 0xF0) == K_SPAN)
     ch = chunkish.reshape(-1, cp) if s.pages % cp == 0 else None
+    # a span is a whole chunk: its head page first, then span tails only
+    for p in np.nonzero((s.kind & 0xF0) == K_SPAN)[0]:
+        if p % cp or (s.kind[p + 1:p + cp] != K_SPAN_TAIL).any():
+            errs.append(f"span at page {p}: not a whole chunk (head + {cp - 1} tails)")
+    tails = np.nonzero(s.kind == K_SPAN_TAIL)[0]
+    if len(tails) and ((s.kind[tails - tails % cp] & 0xF0) != K_SPAN).any():
+        errs.append("span tail page outside a span")
     if ch is None:
         errs.append("pages not a whole number of chunks")
     else:
@@ -165,14 +183,14 @@ def check(s: Snapshot, require_reclaimed: bool = False) -> list:
             if empty.any():
                 errs.append(f"{int(empty.sum())} empty chunk(s) not reclaimed")
     # class semaphores vs bin bitmaps
-    free_slots = np.zeros(s.ncls, dtype=np.int64)
+    free_slots = np.zeros(s.ncls + s.nspan, dtype=np.int64)
     for p, bits in s.bins.items():
-        c = int(s.kind[p]) & 0x0F
+        c = s.page_class(p)
         nfree = int((~bits).sum())
         free_slots[c] += nfree
         if require_reclaimed and nfree == len(bits):
             errs.append(f"empty bin at page {p} not reclaimed")
-    for c in range(s.ncls):
+    for c in range(s.ncls + s.nspan):
         if s.cls_C[c] != free_slots[c]:
             errs.append(f"class {c}: semaphore C={s.cls_C[c]} but {free_slots[c]} free slots")
         if s.cls_absD[c] != 0:

@@ -37,7 +37,8 @@ class GaError(RuntimeError):
 
 class Layout(ctypes.Structure):
     _fields_ = [(n, ctypes.c_uint32) for n in
-                ("page", "chunk_pages", "min_class", "bin_max", "n_classes", "bitmap_bits")]
+                ("page", "chunk_pages", "min_class", "bin_max", "n_classes", "bitmap_bits",
+                 "n_span_classes", "span_max")]
 
 
 class Stats(ctypes.Structure):

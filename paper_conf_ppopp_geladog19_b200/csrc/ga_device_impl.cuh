@@ -42,7 +42,19 @@ constexpr uint64_t kPage = 1ull << kPageShift;
 constexpr int kChunkShift = 6;                  // 64 pages per chunk (R-10)
 constexpr uint32_t kChunkPages = 1u << kChunkShift;
 constexpr int kChunkOrder = kChunkShift;        // a chunk is a TBuddy block of order 6
-constexpr int kNcls = 8;                        // classes 16 .. 2048 B
+// Size classes with per-arena semaphores.  Bins serve 16 B ..
+// 2 KiB out of one 4 KiB page each.  Spans (a B200 departure, DESIGN.md
+// "Spans") serve 4 KiB .. 64 KiB out of one 64-page chunk each, with the same
+// semaphore / bitmap / collective machinery, so mid sizes stop funnelling
+// through TBuddy's global per-order semaphores; TBuddy keeps chunk supply and
+// every size above the span range.  GA_NSPAN=0 restores the paper's routing.
+#ifndef GA_NSPAN
+#define GA_NSPAN 5
+#endif
+constexpr int kNbin = 8;                        // bin classes 16 .. 2048 B
+constexpr int kNspan = GA_NSPAN;                // span classes 4 KiB .. 2^(11+kNspan) B
+static_assert(kNspan >= 0 && kNspan <= 5, "span classes: 4 KiB .. 64 KiB");
+constexpr int kNcls = kNbin + kNspan;           // classes 0 .. kNcls-1
 constexpr int kMinShift = 4;                    // 16 B minimum class (R-13)
 constexpr int kBinWords = 4;                    // 256-bit slot bitmap per page
 constexpr uint64_t kNull = ~0ull;
@@ -103,7 +115,7 @@ static __device__ __forceinline__ void fence_sc() { __threadfence(); }
 // L2, and the read is issued only after the clearing RMW returned, so no SC fence
 // is needed; 0 uses fence.sc + a relaxed load.
 #ifndef GA_RECHECK_RMW
-#define GA_RECHECK_RMW 1
+#define GA_RECHECK_RMW 0
 #endif
 static __device__ __forceinline__ uint64_t recheck_read(uint64_t* p) {
 #if GA_RECHECK_RMW
@@ -175,7 +187,10 @@ static __device__ __forceinline__ uint32_t nth_set(uint64_t x, uint32_t n) {
     return pos;
 }
 
-static __device__ __forceinline__ uint32_t slots_of(int c) { return 256u >> c; }
+static __device__ __forceinline__ bool is_span(int c) { return c >= kNbin; }
+static __device__ __forceinline__ uint32_t slots_of(int c) { return c < kNbin ? 256u >> c : kChunkPages >> (c - kNbin); }
+// first page of the bin / span holding page p (its slot bitmap and kind live there)
+static __device__ __forceinline__ uint64_t bin_head(uint64_t p, int c) { return is_span(c) ? p & ~(uint64_t)(kChunkPages - 1) : p; }
 static __device__ __forceinline__ int words_of(int c) { return c == 0 ? 4 : c == 1 ? 2 : 1; }
 static __device__ __forceinline__ uint64_t valid_mask(int c, int w) {
     int s = (int)slots_of(c) - 64 * w;
@@ -672,8 +687,14 @@ static __device__ __noinline__ void chunk_release(const ga_desc* h, uint64_t ch)
 
 // Make page p a bin of class c for arena A; the caller keeps slots [0, take),
 // the others are opened (the bitmap is all ones while p is not a bin).
+static __device__ __forceinline__ void st_kinds_span(const ga_desc* h, uint64_t head, uint32_t k) {
+    uint32_t* kp = &h->kind[head];                          // 64 u32 = 16 x 16-byte stores
+    for (int i = 0; i < (int)kChunkPages; i += 4)
+        asm volatile("st.relaxed.gpu.global.v4.u32 [%0], {%1,%1,%1,%1};" :: "l"(kp + i), "r"(k) : "memory");
+}
 static __device__ __forceinline__ void bin_init(const ga_desc* h, uint64_t p, uint32_t A, int c, uint32_t take) {
-    st_rlx32(&h->kind[p], kind_bin(A, c));
+    if (is_span(c)) st_kinds_span(h, p, kind_bin(A, c));    // free() looks up any page of the span
+    else st_rlx32(&h->kind[p], kind_bin(A, c));
     fence();
     uint64_t* bw = page_bits(h, p);
     for (int w = 0; w < words_of(c); w++) {
@@ -759,6 +780,17 @@ static __device__ __noinline__ uint64_t bin_find_chunk(const ga_desc* h, uint32_
 // it; threads blocked in a semaphore wait, growers about to take a new chunk,
 // failing mallocs and ga_heap_quiesce do the reclaiming.
 // ---------------------------------------------------------------------------
+// An empty span's chunk back to TBuddy (its slots were taken by the reclaimer;
+// chunk_used stays all ones, as for any chunk outside an arena).
+static __device__ __noinline__ void span_release(const ga_desc* h, uint64_t ch, uint32_t A) {
+    st_kinds_span(h, ch * kChunkPages, 0);
+    if (a_exch(&h->chunk_cand[ch], 0)) hb3_clear_summarised(arena_hb(h, A, kAhbCnd), ch, &h->chunk_cand[ch], 0);
+    st_rlx32(&h->chunk_owner[ch], 0);
+    fence();
+    stat_add(h, kStatChunkReclaim, 1);
+    tree_free(h, kChunkOrder, ch);
+}
+
 // Reclaim page p if it is an empty bin: try-wait all its slots (R-22), then take
 // every slot word with a CAS (all free -> all ones).  `keep`: leave at least
 // that many free slots of the class behind -- delegated reclamation must not
@@ -768,11 +800,13 @@ static __device__ __noinline__ bool bin_reclaim(const ga_desc* h, uint64_t p, ui
     if ((k & 0xC0000000u) != kKindBin) return false;
     uint32_t A = (k >> 8) & 0xFFFFu;
     int c = (int)(k & 0xFF);
+    if (is_span(c) && (p & (kChunkPages - 1))) return false;   // spans: the head page only
     uint64_t* bw = page_bits(h, p);
     uint64_t w[4];
     ld_bitmap(bw, w);
     for (int i = 0; i < words_of(c); i++) if (w[i] & valid_mask(c, i)) return false;
     uint32_t slots = slots_of(c);
+    if (is_span(c) && keep > slots) keep = slots;             // delegated: keep one span's worth
     if (!bsem_trywait(sem_ptr(h, A, c), slots, keep)) return false;
     int i = 0;
     for (; i < words_of(c); i++) {
@@ -788,9 +822,10 @@ static __device__ __noinline__ bool bin_reclaim(const ga_desc* h, uint64_t p, ui
     uint64_t* nf = nonfull_word(h, ch, c);
     uint64_t bit = 1ull << (p & (kChunkPages - 1));
     if (a_and(nf, ~bit) == bit) hb3_clear_summarised(arena_hb(h, A, kAhbNfc + c), ch, nf, 0);
+    stat_add(h, kStatBinReclaim, 1);
+    if (is_span(c)) { span_release(h, ch, A); return true; }
     st_rlx32(&h->kind[p], 0);
     fence();
-    stat_add(h, kStatBinReclaim, 1);
     page_release(h, p);
     return true;
 }
@@ -874,7 +909,7 @@ static __device__ __forceinline__ int size_key(const ga_desc* h, uint64_t n) {
     if (n == 0 || n > (h->pages << kPageShift)) return -1;             // R-15
     if (n <= 16) return 0;
     int lg = 64 - __clzll((long long)(n - 1));                         // ceil(log2 n), R-14
-    if (lg <= 11) return lg - kMinShift;                               // <= 2048 B: bins (R-12)
+    if (lg <= 11 + kNspan) return lg - kMinShift;                      // <= 2048 B: bins (R-12); spans
     int o = lg - kPageShift;
     if (o > (int)h->L) return -1;
     return kNcls + o;
@@ -895,7 +930,42 @@ static __device__ __noinline__ uint64_t bin_claim_one(const ga_desc* h, uint32_t
         if (got) return (p << kPageShift) + (uint64_t)(wi * 64 + __ffsll((long long)got) - 1) * csz;
     }
 }
+// a fresh span for arena A straight from TBuddy (one chunk); -1 if the tree is exhausted
+static __device__ __noinline__ int64_t span_acquire(const ga_desc* h, uint32_t A) {
+    int64_t ch = tree_alloc_one_retry(h, kChunkOrder);
+    if (ch < 0) return -1;
+    st_rlx32(&h->chunk_owner[ch], A + 1);
+    stat_add(h, kStatChunkGrow, 1);
+    return ch;
+}
+static __device__ __noinline__ uint64_t span_malloc_lane(const ga_desc* h, uint32_t A0, int c) {
+    uint32_t slots = slots_of(c);
+    for (int attempt = 0; attempt < 2; attempt++) {
+        if (bsem_wait(sem_ptr(h, A0, c), 1, slots, ArenaSpin{h, A0}) == kAcquired) return bin_claim_one(h, A0, c);
+        reclaim_arena(h, A0, -1, kReclaimKeep);
+        int64_t ch = span_acquire(h, A0);
+        if (ch >= 0) {
+            uint64_t p = (uint64_t)ch * kChunkPages;
+            bin_init(h, p, A0, c, 1);
+            stat_add(h, kStatBinGrow, 1);
+            st_rlx32(&h->hint[A0 * kNcls + c], (uint32_t)p);
+            bsem_signal(sem_ptr(h, A0, c), slots - 1, slots - 1);
+            return p << kPageShift;
+        }
+        bsem_signal(sem_ptr(h, A0, c), 0, slots - 1);
+        if (attempt == 0) reclaim_all(h);
+    }
+    for (uint32_t t = 1; t <= h->n_arenas; t++) {
+        uint32_t B = (A0 + t) % h->n_arenas;
+        uint64_t cw = ld_rlx(sem_ptr(h, B, c));
+        if (sem_C(cw) < 1 && (int64_t)sem_C(cw) + sem_D(cw) < 1) continue;
+        if (bsem_wait(sem_ptr(h, B, c), 1, 1, NoSpin()) == kAcquired) return bin_claim_one(h, B, c);
+    }
+    stat_add(h, kStatFail, 1);
+    return kNull;
+}
 static __device__ __noinline__ uint64_t bin_malloc_lane(const ga_desc* h, uint32_t A0, int c) {
+    if (is_span(c)) return span_malloc_lane(h, A0, c);
     uint32_t slots = slots_of(c);
     for (int attempt = 0; attempt < 2; attempt++) {
         if (bsem_wait(sem_ptr(h, A0, c), 1, slots, ArenaSpin{h, A0}) == kAcquired) return bin_claim_one(h, A0, c);
@@ -1043,6 +1113,51 @@ static __device__ __noinline__ uint64_t bin_grow_collective(const ga_desc* h, un
     return my;
 }
 
+// ---- spans: collective growth (class semaphore said GROW for the group) ------
+// ceil(N/slots) fresh chunks straight from TBuddy, one at a time: the leader
+// takes a chunk, lanes [served, served + take) get its slots and the first of
+// them initialises the span.  If the tree runs dry the lanes served so far
+// keep their slots, the others get kNull (the caller degrades them to per-lane
+// waits) and the unproduced units are retracted (signal(0, B'-N)).
+static __device__ __noinline__ uint64_t span_grow_collective(const ga_desc* h, unsigned grp, uint32_t A, int c) {
+    const uint32_t lane = lane_id();
+    const int leader = __ffs(grp) - 1;
+    const uint32_t N = __popc(grp), rank = __popc(grp & lanemask_lt());
+    const uint32_t slots = slots_of(c);
+    const uint32_t Bp = slots * ((N + slots - 1) / slots);                 // R-8
+    const uint64_t csz = 16ull << c;
+    uint64_t my = kNull;
+    uint32_t served = 0;
+    int64_t ch = 0;
+    while (served < N) {
+        if ((int)lane == leader) {
+            if (served == 0) reclaim_arena(h, A, -1, kReclaimKeep);       // delegated work first
+            ch = span_acquire(h, A);
+        }
+        ch = __shfl_sync(grp, ch, leader);
+        if (ch < 0) break;
+        const uint32_t take = N - served < slots ? N - served : slots;
+        const uint64_t p = (uint64_t)ch * kChunkPages;
+        if (rank >= served && rank < served + take) {
+            const uint32_t r = rank - served;
+            my = (p << kPageShift) + (uint64_t)r * csz;
+            if (r == 0) bin_init(h, p, A, c, take);
+        }
+        served += take;
+    }
+    __syncwarp(grp);
+    if ((int)lane == leader) {
+        stat_add(h, kStatBinGrow, (served + slots - 1) / slots);
+        if (ch >= 0) {
+            st_rlx32(&h->hint[A * kNcls + c], (uint32_t)((uint64_t)ch * kChunkPages));
+            bsem_signal(sem_ptr(h, A, c), Bp - N, Bp - N);                  // release: spans initialised
+        } else {
+            bsem_signal(sem_ptr(h, A, c), 0, Bp - N);                       // failure
+        }
+    }
+    return my;
+}
+
 // ---- TBuddy, group path -------------------------------------------------------
 // One bulk wait of N units per order for the group (batch 2, B' = 2*ceil(N/2));
 // on GROW the group climbs with N_{k+1} = ceil(N_k / 2), claims N_m nodes at the
@@ -1131,7 +1246,8 @@ static __device__ __noinline__ uint64_t ga_malloc_off(const ga_desc* h, uint64_t
         if ((int)lane_id() == leader)
             r = bsem_wait(sem_ptr(h, A, key), N, slots * ((N + slots - 1) / slots), ArenaSpin{h, A});
         r = __shfl_sync(grp, r, leader);
-        my = r == kAcquired ? bin_claim_collective(h, grp, A, key) : bin_grow_collective(h, grp, A, key);
+        my = r == kAcquired ? bin_claim_collective(h, grp, A, key)
+           : is_span(key) ? span_grow_collective(h, grp, A, key) : bin_grow_collective(h, grp, A, key);
         if (__any_sync(grp, my == kNull)) {                 // R-27: degrade to per-lane waits
             if ((int)lane_id() == leader) stat_add(h, kStatFallback, 1);
             if (my == kNull) my = bin_malloc_lane(h, A, key);
@@ -1189,7 +1305,8 @@ static __device__ __noinline__ void ga_free_off(const ga_desc* h, uint64_t off) 
     if (!is_bin) return;
     const uint32_t A = (k >> 8) & 0xFFFFu;
     const int c = (int)(k & 0xFF);
-    const uint32_t slot = (uint32_t)((off & (kPage - 1)) >> (c + kMinShift));
+    p = bin_head(p, c);                                        // spans: bitmap at the chunk's first page
+    const uint32_t slot = (uint32_t)((off - (p << kPageShift)) >> (c + kMinShift));
     const int w = (int)(slot >> 6);
     const unsigned g1 = __match_any_sync(bins, (p << 2) | (uint64_t)w);
     const uint64_t bit = 1ull << (slot & 63);
@@ -1208,7 +1325,7 @@ static __device__ __noinline__ void ga_free_off(const ga_desc* h, uint64_t off) 
         }
     }
     __syncwarp(bins);
-    const unsigned g2 = __match_any_sync(bins, (A << 3) | (uint32_t)c);
+    const unsigned g2 = __match_any_sync(bins, (A << 4) | (uint32_t)c);     // class < 16
     if ((int)lane_id() == __ffs(g2) - 1) bsem_signal_after_rmw(sem_ptr(h, A, c), __popc(g2));
 }
 

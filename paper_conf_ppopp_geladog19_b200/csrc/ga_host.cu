@@ -111,9 +111,11 @@ ga_status ga_layout(ga_layout_t* out) {
     out->page = (uint32_t)kPage;
     out->chunk_pages = kChunkPages;
     out->min_class = 1u << kMinShift;
-    out->bin_max = 1u << (kMinShift + kNcls - 1);
-    out->n_classes = kNcls;
+    out->bin_max = 1u << (kMinShift + kNbin - 1);
+    out->n_classes = kNbin;
     out->bitmap_bits = 64 * kBinWords;
+    out->n_span_classes = kNspan;
+    out->span_max = kNspan ? (uint32_t)kPage << (kNspan - 1) : 0;
     return GA_OK;
 }
 
@@ -328,7 +330,7 @@ ga_status ga_heap_snapshot(ga_heap_t h, ga_stream_t stream, void* host, size_t c
     put64(d.pages * kPage);
     put64(d.pages);
     put64(kPage | ((uint64_t)(d.L + 1) << 32));
-    put64((1ull << kMinShift) | ((uint64_t)kNcls << 32) | ((uint64_t)kChunkPages << 48));
+    put64((1ull << kMinShift) | ((uint64_t)kNbin << 32) | ((uint64_t)kNspan << 40) | ((uint64_t)kChunkPages << 48));
     std::vector<uint8_t> kb(d.pages, 0x00);
     for (uint32_t n = 0; n <= d.L; n++) {
         uint64_t cnt = 1ull << (d.L - n);
@@ -346,16 +348,18 @@ ga_status ga_heap_snapshot(ga_heap_t h, ga_stream_t stream, void* host, size_t c
         if (!owner[ch]) continue;
         for (uint32_t j = 0; j < kChunkPages; j++) {
             uint64_t p = ch * kChunkPages + j;
+            const uint32_t c = kind[p] & 0xFF;
             if (!((used_[ch] >> j) & 1)) kb[p] = 0x02;
-            else if ((kind[p] & 0xC0000000u) == kKindBin) kb[p] = (uint8_t)(0x10 | (kind[p] & 0xFF));
+            else if ((kind[p] & 0xC0000000u) == kKindBin && c < (uint32_t)kNbin) kb[p] = (uint8_t)(0x10 | c);
+            else if ((kind[p] & 0xC0000000u) == kKindBin) kb[p] = (uint8_t)(j == 0 ? 0x20 | (c - kNbin) : 0x04);
             else kb[p] = 0xFF;                              // claimed page that is not a bin: not quiescent
         }
     }
     put(kb.data(), kb.size());
     for (uint64_t p = 0; p < d.pages; p++) {
-        if ((kb[p] & 0xF0) != 0x10 || kb[p] == 0xFF) continue;
-        int c = kb[p] & 0x0F;
-        uint32_t slots = 256u >> c;
+        if (((kb[p] & 0xF0) != 0x10 && (kb[p] & 0xF0) != 0x20) || kb[p] == 0xFF) continue;
+        int c = (kb[p] & 0x0F) + ((kb[p] & 0xF0) == 0x20 ? kNbin : 0);
+        uint32_t slots = c < kNbin ? 256u >> c : kChunkPages >> (c - kNbin);
         uint8_t tmp[32] = {0};
         for (uint32_t sl = 0; sl < slots; sl++)
             if ((bits[p * kBinWords + sl / 64] >> (sl % 64)) & 1) tmp[sl / 8] |= (uint8_t)(1u << (sl % 8));
