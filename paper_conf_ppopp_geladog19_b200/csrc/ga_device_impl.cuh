@@ -55,6 +55,16 @@ constexpr int kNbin = 8;                        // bin classes 16 .. 2048 B
 constexpr int kNspan = GA_NSPAN;                // span classes 4 KiB .. 2^(11+kNspan) B
 static_assert(kNspan >= 0 && kNspan <= 5, "span classes: 4 KiB .. 64 KiB");
 constexpr int kNcls = kNbin + kNspan;           // classes 0 .. kNcls-1
+// Span arenas are shared by GA_SPAN_SHARE consecutive SMs: fewer, larger pools
+// smooth the per-pool high-water marks that set reserved memory (DESIGN.md
+// "Spans").  GA_SPAN_EAGER=1: a free that empties a span returns it to the
+// tree at once when the class keeps a span's worth of free slots elsewhere.
+#ifndef GA_SPAN_SHARE
+#define GA_SPAN_SHARE 4
+#endif
+#ifndef GA_SPAN_EAGER
+#define GA_SPAN_EAGER 1
+#endif
 constexpr int kMinShift = 4;                    // 16 B minimum class (R-13)
 constexpr int kBinWords = 4;                    // 256-bit slot bitmap per page
 constexpr uint64_t kNull = ~0ull;
@@ -564,6 +574,22 @@ static __device__ __noinline__ bool tree_has_supply(const ga_desc* h, int o, boo
 // 5. UAlloc: chunks of 64 pages owned by one arena, one-page bins
 // ---------------------------------------------------------------------------
 static __device__ __forceinline__ uint32_t kind_bin(uint32_t A, int c) { return kKindBin | (A << 8) | (uint32_t)c; }
+// Clear bit ch of one of arena A's chunk summaries when chunk ch is no longer
+// A's or its data word reads `empty_value`; re-check both after the clear
+// (clear-then-recheck).  A chunk that left A for another arena (spans recycle
+// chunks often) must not stay visible in A's summary, or A's searches would
+// keep returning it.
+static __device__ __noinline__ void hb3_clear_owned(const ga_desc* h, HB3 b, uint64_t ch, uint32_t A,
+                                                    const uint64_t* data, uint64_t empty_value) {
+    uint64_t bit = 1ull << (ch & 63);
+    uint64_t old = a_and(&b.w0[ch >> 6], ~bit);
+    fence_sc();
+    if (ld_rlx32(&h->chunk_owner[ch]) == A + 1 && ld_rlx(data) != empty_value) {
+        if (a_or(&b.w0[ch >> 6], bit) == 0) hb3_up_set(b, (uint32_t)(ch >> 6));
+        return;
+    }
+    if (old == bit) hb3_up_clear(b, (uint32_t)(ch >> 6));
+}
 static __device__ __forceinline__ uint64_t* nonfull_word(const ga_desc* h, uint64_t ch, int c) { return &h->chunk_nonfull[ch * kNcls + c]; }
 static __device__ __forceinline__ bool page_full(const uint64_t w[4], int c) {
     for (int i = 0; i < words_of(c); i++) if ((w[i] | ~valid_mask(c, i)) != ~0ull) return false;
@@ -597,11 +623,15 @@ static __device__ __noinline__ void nonfull_clear_if_full(const ga_desc* h, uint
     fence_sc();
     ld_bitmap(page_bits(h, p), w);
 #endif
-    if (ld_rlx32(&h->kind[p]) == kind_bin(A, c) && !page_full(w, c)) {
-        if (a_or(nf, bit) == 0) hb3_set(arena_hb(h, A, kAhbNfc + c), ch);
+    // Re-set the bit if p is a non-full class-c bin of ANY arena: a stale caller
+    // (its chunk went back to the tree and on to another arena, which made p a
+    // class-c bin again) must not leave the new owner's bin invisible.
+    const uint32_t k = ld_rlx32(&h->kind[p]);
+    if ((k & 0xC0000000u) == kKindBin && (int)(k & 0xFF) == c && !page_full(w, c)) {
+        if (a_or(nf, bit) == 0) hb3_set(arena_hb(h, (k >> 8) & 0xFFFFu, kAhbNfc + c), ch);
         return;
     }
-    if (old == bit) hb3_clear_summarised(arena_hb(h, A, kAhbNfc + c), ch, nf, 0);
+    if (old == bit) hb3_clear_owned(h, arena_hb(h, A, kAhbNfc + c), ch, A, nf, 0);
 }
 
 // Take a new chunk from TBuddy for arena A, keep its first k pages, open the rest.
@@ -633,6 +663,10 @@ static __device__ __noinline__ uint64_t page_claim(const ga_desc* h, uint32_t A,
                 uint32_t bit = first_from(cm, seed);
                 cm &= ~(1ull << bit);
                 uint64_t ch = (uint64_t)j * 64 + bit;
+                if (ld_rlx32(&h->chunk_owner[ch]) != A + 1) {        // left the arena: stale bit
+                    hb3_clear_owned(h, fb, ch, A, &h->chunk_used[ch], ~0ull);
+                    continue;
+                }
                 uint64_t u = ld_rlx(&h->chunk_used[ch]);
                 while (~u) {
                     uint64_t m = lowest_bits(~u, need);
@@ -739,15 +773,54 @@ static __device__ __noinline__ uint64_t bin_claim_page(const ga_desc* h, uint64_
     return 0;
 }
 
+#if GA_DEBUG
+// Debug builds: a claimer stuck in bin_find_chunk audits arena A's class-c
+// bins once (single auditor) into the debug header words 1..7.
+static __device__ __noinline__ void nfc_audit(const ga_desc* h, uint32_t A, int c) {
+    uint64_t* dbg = g_ga_dbg;
+    if (!dbg || atomicCAS((unsigned long long*)&dbg[1], 0ull, 1ull) != 0ull) return;
+    HB3 nb = arena_hb(h, A, kAhbNfc + c);
+    uint64_t nbins = 0, nfree = 0, lost_nf = 0, lost_sum = 0, lost_up = 0;
+    for (uint64_t ch = 0; ch < h->nchunks; ch++) {
+        if (ld_rlx32(&h->chunk_owner[ch]) != A + 1) continue;
+        uint64_t nf = ld_rlx(nonfull_word(h, ch, c));
+        for (uint32_t j = 0; j < kChunkPages; j++) {
+            uint64_t p = ch * kChunkPages + j;
+            if (ld_rlx32(&h->kind[p]) != kind_bin(A, c) || bin_head(p, c) != p) continue;
+            nbins++;
+            uint64_t w[4];
+            ld_bitmap(page_bits(h, p), w);
+            uint64_t fr = 0;
+            for (int i = 0; i < words_of(c); i++) fr += __popcll(~w[i] & valid_mask(c, i));
+            nfree += fr;
+            if (fr && !((nf >> j) & 1)) lost_nf++;
+        }
+        if (nf) {
+            if (!((ld_rlx(&nb.w0[ch >> 6]) >> (ch & 63)) & 1)) lost_sum++;
+            else if (!((ld_rlx(&hb3_w1(nb)[ch >> 12]) >> ((ch >> 6) & 63)) & 1) ||
+                     !((ld_rlx(&hb3_w2(nb)[ch >> 18]) >> ((ch >> 12) & 63)) & 1)) lost_up++;
+        }
+    }
+    uint64_t sw = ld_rlx(sem_ptr(h, A, c));
+    volatile uint64_t* r = (volatile uint64_t*)dbg;
+    r[2] = ((uint64_t)A << 8) | (uint64_t)c | ((uint64_t)(uint32_t)sem_C(sw) << 32);
+    r[3] = nbins; r[4] = nfree; r[5] = lost_nf; r[6] = lost_sum;
+    r[7] = lost_up | ((uint64_t)(uint32_t)sem_D(sw) << 32);
+    __threadfence_system();
+    r[1] = 2;
+}
+#endif
+
 // A chunk of arena A with non-full class-c bins, and its non-full page mask:
 // the hint's chunk first, then the (A, c) summary.  Spins until one shows up
 // (the caller holds units, so a free slot exists or is being published).
 static __device__ __noinline__ uint64_t bin_find_chunk(const ga_desc* h, uint32_t A, int c, uint64_t* mask_out) {
     GA_DBG_CNT;
     uint32_t hp = ld_rlx32(&h->hint[A * kNcls + c]);
-    if (hp < h->pages) {
+    if (hp < h->pages) {                                      // the hint's chunk, if still A's
+        const uint32_t own = ld_rlx32(&h->chunk_owner[hp >> kChunkShift]);
         uint64_t m = ld_rlx(nonfull_word(h, hp >> kChunkShift, c));
-        if (m) { *mask_out = m; return hp >> kChunkShift; }
+        if (own == A + 1 && m) { *mask_out = m; return hp >> kChunkShift; }
     }
     HB3 nb = arena_hb(h, A, kAhbNfc + c);
     uint32_t seed = scatter_seed();
@@ -760,15 +833,19 @@ static __device__ __noinline__ uint64_t bin_find_chunk(const ga_desc* h, uint32_
                 uint32_t bit = first_from(cm, seed);
                 cm &= ~(1ull << bit);
                 uint64_t ch = (uint64_t)j * 64 + bit;
+                const uint32_t own = ld_rlx32(&h->chunk_owner[ch]);
                 uint64_t m = ld_rlx(nonfull_word(h, ch, c));
-                if (m) {
+                if (own == A + 1 && m) {
                     st_rlx32(&h->hint[A * kNcls + c], (uint32_t)(ch * kChunkPages + (__ffsll((long long)m) - 1)));
                     *mask_out = m;
                     return ch;
                 }
-                hb3_clear_summarised(nb, ch, nonfull_word(h, ch, c), 0);    // stale summary bit
+                hb3_clear_owned(h, nb, ch, A, nonfull_word(h, ch, c), 0);    // stale summary bit
             }
         }
+#if GA_DEBUG
+        if (((dbg_cnt + 1) & ((1u << 18) - 1)) == 0) nfc_audit(h, A, c);
+#endif
         SPIN_NOTE(dbg_cnt, 7, ((uint64_t)A << 8) | c, ns);
         __nanosleep(ns); if (ns < 1024) ns <<= 1;
         seed = hash32(seed + 7);
@@ -821,7 +898,7 @@ static __device__ __noinline__ bool bin_reclaim(const ga_desc* h, uint64_t p, ui
     uint64_t ch = p >> kChunkShift;
     uint64_t* nf = nonfull_word(h, ch, c);
     uint64_t bit = 1ull << (p & (kChunkPages - 1));
-    if (a_and(nf, ~bit) == bit) hb3_clear_summarised(arena_hb(h, A, kAhbNfc + c), ch, nf, 0);
+    if (a_and(nf, ~bit) == bit) hb3_clear_owned(h, arena_hb(h, A, kAhbNfc + c), ch, A, nf, 0);
     stat_add(h, kStatBinReclaim, 1);
     if (is_span(c)) { span_release(h, ch, A); return true; }
     st_rlx32(&h->kind[p], 0);
@@ -1239,7 +1316,7 @@ static __device__ __noinline__ uint64_t ga_malloc_off(const ga_desc* h, uint64_t
     if (key < 0) return kNull;
     uint64_t my;
     if (key < kNcls) {
-        const uint32_t A = arena_of(h);
+        const uint32_t A = is_span(key) ? arena_of(h) / GA_SPAN_SHARE : arena_of(h);
         const uint32_t N = __popc(grp), slots = slots_of(key);
         const int leader = __ffs(grp) - 1;
         int r = 0;
@@ -1311,6 +1388,7 @@ static __device__ __noinline__ void ga_free_off(const ga_desc* h, uint64_t off) 
     const unsigned g1 = __match_any_sync(bins, (p << 2) | (uint64_t)w);
     const uint64_t bit = 1ull << (slot & 63);
     const uint64_t mask = ((uint64_t)__reduce_or_sync(g1, (uint32_t)(bit >> 32)) << 32) | __reduce_or_sync(g1, (uint32_t)bit);
+    bool eager = false;
     if ((int)lane_id() == __ffs(g1) - 1) {
         uint64_t* bw = page_bits(h, p);
         const uint64_t old = a_and(&bw[w], ~mask);
@@ -1321,12 +1399,19 @@ static __device__ __noinline__ void ga_free_off(const ga_desc* h, uint64_t off) 
             ld_bitmap(bw, ww);
             bool empty = true;
             for (int i = 0; i < words_of(c); i++) if (ww[i] & valid_mask(c, i)) empty = false;
-            if (empty) mark_candidate(h, p, A);
+            if (empty) {
+                if (GA_SPAN_EAGER && is_span(c)) eager = true;   // reclaim after the signal below
+                else mark_candidate(h, p, A);
+            }
         }
     }
     __syncwarp(bins);
     const unsigned g2 = __match_any_sync(bins, (A << 4) | (uint32_t)c);     // class < 16
     if ((int)lane_id() == __ffs(g2) - 1) bsem_signal_after_rmw(sem_ptr(h, A, c), __popc(g2));
+    if (eager) {
+        fence();                                               // our slots' units are published
+        if (!bin_reclaim(h, p, slots_of(c))) mark_candidate(h, p, A);
+    }
 }
 
 }  // namespace ga
