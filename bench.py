@@ -115,6 +115,37 @@ def oracle_leg(trace, budget_s: float = 10.0) -> dict:
             "seconds": t_total, "stats": st}
 
 
+def _oracle_shard(arg):
+    sizes, heap_bytes, D, budget_s = arg
+    import oracle
+    calls, t_total, runs = 0, 0.0, 0
+    while t_total < budget_s or runs == 0:
+        t0 = time.perf_counter()
+        r = oracle.run_trace(sizes, heap_bytes, D, want_ok=False)
+        t_total += time.perf_counter() - t0
+        calls += r.stats["calls"]
+        runs += 1
+    return calls, t_total
+
+
+def oracle_leg_parallel(trace, budget_s: float = 6.0) -> dict:
+    """SURVEY.md 8(d) "P cores": P = usable host cores independent oracle instances,
+    instance j on the threads tid = j mod P with a heap/P heap (rounded down to a
+    chunk multiple); the aggregate of their calls/s."""
+    import multiprocessing as mp
+    import oracle
+    oracle.build()
+    P = max(1, min(cpu_cores(), 64))
+    hb = max(256 << 10, (trace.heap_bytes // P) & ~((256 << 10) - 1))
+    shards = [(np.ascontiguousarray(trace.sizes[:, j::P]), hb, trace.D, budget_s) for j in range(P)]
+    with mp.get_context("fork").Pool(P) as pool:
+        out = pool.map(_oracle_shard, shards)
+    value = sum(c / t for c, t in out)
+    return {"value": value, "unit": UNIT, "cores": P, "kind": "oracle",
+            "sample": f"{trace.name}: {P} independent sequential C oracles, shard j = threads tid = j mod {P}, "
+                      f"heap {hb} B each, each repeated for ~{budget_s:.0f} s"}
+
+
 # ----------------------------------------------------------------------------- reference arm
 def run_reference(args, trace):
     rank = int(os.environ.get("RANK", "0"))
@@ -183,6 +214,50 @@ def d3_sweep(ga, heap, stream, dev, T, args, sizes=(16, 32, 64, 128, 256, 512, 1
     vals = [v["speedup"] for v in res.values()]
     res["min_speedup"] = min(vals)
     res["geomean_speedup"] = float(np.exp(np.mean(np.log(vals))))
+    return res
+
+
+def d4_levels(ga, stream, dev, args, flush, levels=("fit", "exhaust"), reps=3):
+    """d4 at the other two pressure levels: the same mixed trace on
+    a 16 GiB heap (fit: every malloc succeeds) and a 3 GiB heap (exhaust: ~95 %
+    rounded-live, failures and deferred reclamation).  calls/s from the timed
+    kernel; failures and fragmentation from correctness mode, beside the oracle's."""
+    import torch
+    import oracle
+    from paper_conf_ppopp_geladog19_b200.runner import GpuHeap, run_correctness
+    oracle.build()
+    res = {}
+    cc = torch.zeros(8, dtype=torch.int64, device=dev)
+    for lv in levels:
+        t = tracegen.d4_mixed(lv)
+        heap = GpuHeap(t.heap_bytes, device=dev.index or 0, stream=stream)
+        d = torch.from_numpy(t.sizes.view(np.int32)).to(dev)
+        times, fails = [], 0
+        for rep in range(reps + 1):
+            flush.fill_(rep)
+            cc.zero_()
+            a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a0.record(stream)
+            ga.ga_trace_timed(heap.h, stream.cuda_stream, d.data_ptr(), t.R, t.T, t.D, cc.data_ptr(), args.block)
+            a1.record(stream)
+            a1.synchronize()
+            if rep:
+                times.append(a0.elapsed_time(a1) / 1e3)
+                fails = max(fails, int(cc[1].item()))
+        calls = int(cc[0].item() + cc[2].item())
+        heap.reset()
+        run = run_correctness(heap, t.sizes, t.D, log=False, tag=False, reserved=True)
+        ref = oracle.run_trace(t.sizes, t.heap_bytes, t.D, want_ok=False).stats
+        fg = run.peak_reserved_bytes / run.peak_live_bytes if run.peak_live_bytes else None
+        fo = ref["peak_reserved_bytes"] / ref["peak_live_bytes"]
+        st = heap.stats()
+        res[lv] = {"heap_bytes": t.heap_bytes, "calls_per_s": calls / (sum(times) / len(times)),
+                   "ms": sum(times) / len(times), "timed_failed_mallocs": fails,
+                   "correctness_failed_mallocs": run.counts["n_fail"], "oracle_failed_mallocs": ref["n_malloc_fail"],
+                   "fragmentation": {"gpu": fg, "oracle": fo, "ratio": fg / fo if fg else None},
+                   "stats": {k: int(v) for k, v in st.items() if isinstance(v, (int, np.integer))}}
+        heap.close()
+        del d
     return res
 
 
@@ -381,6 +456,7 @@ def main():
         cpu.pop("stats")
         cpu.pop("seconds")
         out["cpu_baseline"] = cpu
+        out["cpu_baseline_all_cores"] = oracle_leg_parallel(trace)
 
         # ---- CUDA device malloc on the same trace (bounded prefix of rounds)
         heap.reset()
@@ -408,6 +484,9 @@ def main():
         # ---- d3: warp-uniform sizes 16 B - 8 KiB (BASELINE configs[2]), malloc+free per
         # thread and round (D = 0), full grid; CUDA malloc on a bounded prefix of rounds
         out["d3_sweep"] = d3_sweep(ga, heap, stream, dev, T, args)
+
+        # ---- d4 at the fit and exhaust pressure levels
+        out["d4_levels"] = d4_levels(ga, stream, dev, args, flush)
 
         # ---- d2: bulk-semaphore microbenchmark (BASELINE configs[1], Sec. 5.1)
         out["d2_bsem"] = d2_bsem(ga, stream, dev)

@@ -592,7 +592,8 @@ static __device__ __noinline__ void hb3_clear_owned(const ga_desc* h, HB3 b, uin
 }
 static __device__ __forceinline__ uint64_t* nonfull_word(const ga_desc* h, uint64_t ch, int c) { return &h->chunk_nonfull[ch * kNcls + c]; }
 static __device__ __forceinline__ bool page_full(const uint64_t w[4], int c) {
-    for (int i = 0; i < words_of(c); i++) if ((w[i] | ~valid_mask(c, i)) != ~0ull) return false;
+#pragma unroll
+    for (int i = 0; i < 4; i++) if (i < words_of(c)) if ((w[i] | ~valid_mask(c, i)) != ~0ull) return false;
     return true;
 }
 
@@ -603,12 +604,23 @@ struct ArenaSpin {
     __device__ void operator()() const { reclaim_arena(h, A, 4, kReclaimKeep); }
 };
 
+// Data bit `bit` of *data (a per-chunk word: non-full pages, reclaim
+// candidates) goes up, and chunk ch must then be visible in summary b.  The
+// data word can hold a stale bit from the chunk's previous life (a free's
+// delayed publication that landed after the page was reclaimed, while a stale
+// summary bit was being cleaned up under another owner), so "the word was
+// already non-zero" does not prove the summary has ch: the summary bit is
+// checked after the data RMW has performed (a clearer re-checks the data after
+// its own clear, so one of the two always sees the other).
+static __device__ __noinline__ void summarised_set(HB3 b, uint64_t ch, uint64_t* data, uint64_t bit) {
+    const uint64_t cb = 1ull << (ch & 63);
+    if ((ld_rlx(data) & bit) == bit && (ld_rlx(&b.w0[ch >> 6]) & cb)) return;
+    if (a_or(data, bit) == 0 || !(ld_rlx(&b.w0[ch >> 6]) & cb)) hb3_set(b, ch);
+}
 // page p (class c, arena A) has a free slot again
 static __device__ __forceinline__ void nonfull_set(const ga_desc* h, uint64_t p, int c, uint32_t A) {
-    uint64_t* nf = nonfull_word(h, p >> kChunkShift, c);
-    uint64_t bit = 1ull << (p & (kChunkPages - 1));
-    if (ld_rlx(nf) & bit) return;
-    if (a_or(nf, bit) == 0) hb3_set(arena_hb(h, A, kAhbNfc + c), p >> kChunkShift);
+    summarised_set(arena_hb(h, A, kAhbNfc + c), p >> kChunkShift, nonfull_word(h, p >> kChunkShift, c),
+                   1ull << (p & (kChunkPages - 1)));
 }
 // drop p from the non-full set if it is really full (clear-then-recheck)
 static __device__ __noinline__ void nonfull_clear_if_full(const ga_desc* h, uint64_t p, int c, uint32_t A) {
@@ -628,7 +640,7 @@ static __device__ __noinline__ void nonfull_clear_if_full(const ga_desc* h, uint
     // class-c bin again) must not leave the new owner's bin invisible.
     const uint32_t k = ld_rlx32(&h->kind[p]);
     if ((k & 0xC0000000u) == kKindBin && (int)(k & 0xFF) == c && !page_full(w, c)) {
-        if (a_or(nf, bit) == 0) hb3_set(arena_hb(h, (k >> 8) & 0xFFFFu, kAhbNfc + c), ch);
+        summarised_set(arena_hb(h, (k >> 8) & 0xFFFFu, kAhbNfc + c), ch, nf, bit);
         return;
     }
     if (old == bit) hb3_clear_owned(h, arena_hb(h, A, kAhbNfc + c), ch, A, nf, 0);
@@ -741,14 +753,32 @@ static __device__ __forceinline__ void bin_init(const ga_desc* h, uint64_t p, ui
 }
 
 // Claim up to `need` slots of page p (an (A, c) bin) from one bitmap word with
-// one atomicOr.  Returns the claimed mask (word in *wi); 0 if none.
-static __device__ __noinline__ uint64_t bin_claim_page(const ga_desc* h, uint64_t p, uint32_t A, int c, int need, int* wi) {
-    if (ld_rlx32(&h->kind[p]) != kind_bin(A, c)) return 0;
+// one atomicOr.  Returns the claimed mask (word in *wi); 0 if none.  The page
+// kind and the bitmap are loaded together (independent round trips), and the
+// word scan starts at `rot` so concurrent warps on one page spread over its
+// words (scattered search).  Loops stay rolled: this is the hottest
+// code of the allocator and instruction-fetch stalls dominate.
+static __device__ __noinline__ uint64_t bin_claim_page(const ga_desc* h, uint64_t p, uint32_t A, int c, int need, int* wi,
+                                                       uint32_t rot) {
     uint64_t* bw = page_bits(h, p);
     uint64_t w[4];
+    const uint32_t k0 = ld_rlx32(&h->kind[p]);
     ld_bitmap(bw, w);
-    for (int i = 0; i < words_of(c); i++) {
-        uint64_t fr = ~w[i] & valid_mask(c, i);
+    if (k0 != kind_bin(A, c)) {
+        // A stale non-full bit: a free's delayed nonfull_set can land after the
+        // page was reclaimed (or re-classed).  Drop it (the helper re-sets it if
+        // p is in fact a non-full class-c bin), or every claimer that lands on
+        // p would retry it forever.
+        nonfull_clear_if_full(h, p, c, A);
+        return 0;
+    }
+    const int nw = words_of(c);
+#pragma unroll 1
+    for (int t = 0; t < nw; t++) {
+        const int i = (int)((t + rot) & (uint32_t)(nw - 1));
+        const uint64_t vm = valid_mask(c, i);
+        uint64_t wi_v = i == 0 ? w[0] : i == 1 ? w[1] : i == 2 ? w[2] : w[3];
+        uint64_t fr = ~wi_v & vm;
         while (fr) {
             uint64_t m = lowest_bits(fr, need);
             uint64_t old = a_or(&bw[i], m);
@@ -758,15 +788,14 @@ static __device__ __noinline__ uint64_t bin_claim_page(const ga_desc* h, uint64_
                     a_and(&bw[i], ~got);
                     return 0;
                 }
-                w[i] = old | m;
-                if ((w[i] | ~valid_mask(c, i)) == ~0ull) {         // this word is full now
+                if (((old | m) | ~vm) == ~0ull) {                  // this word is full now
                     ld_bitmap(bw, w);
                     if (page_full(w, c)) nonfull_clear_if_full(h, p, c, A);
                 }
                 *wi = i;
                 return got;
             }
-            fr = ~(old | m) & valid_mask(c, i);
+            fr = ~(old | m) & vm;
         }
     }
     nonfull_clear_if_full(h, p, c, A);
@@ -881,7 +910,8 @@ static __device__ __noinline__ bool bin_reclaim(const ga_desc* h, uint64_t p, ui
     uint64_t* bw = page_bits(h, p);
     uint64_t w[4];
     ld_bitmap(bw, w);
-    for (int i = 0; i < words_of(c); i++) if (w[i] & valid_mask(c, i)) return false;
+#pragma unroll
+    for (int i = 0; i < 4; i++) if (i < words_of(c) && (w[i] & valid_mask(c, i))) return false;
     uint32_t slots = slots_of(c);
     if (is_span(c) && keep > slots) keep = slots;             // delegated: keep one span's worth
     if (!bsem_trywait(sem_ptr(h, A, c), slots, keep)) return false;
@@ -908,10 +938,8 @@ static __device__ __noinline__ bool bin_reclaim(const ga_desc* h, uint64_t p, ui
 }
 
 static __device__ __forceinline__ void mark_candidate(const ga_desc* h, uint64_t p, uint32_t A) {
-    uint64_t* cw = &h->chunk_cand[p >> kChunkShift];
-    uint64_t bit = 1ull << (p & (kChunkPages - 1));
-    if (ld_rlx(cw) & bit) return;
-    if (a_or(cw, bit) == 0) hb3_set(arena_hb(h, A, kAhbCnd), p >> kChunkShift);
+    summarised_set(arena_hb(h, A, kAhbCnd), p >> kChunkShift, &h->chunk_cand[p >> kChunkShift],
+                   1ull << (p & (kChunkPages - 1)));
 }
 
 // Reclaim up to `budget` candidate bins of arena A (budget < 0: all), leaving
@@ -940,14 +968,15 @@ static __device__ __noinline__ void reclaim_arena(const ga_desc* h, uint32_t A, 
                 if (ld_rlx32(&h->kind[ch * kChunkPages + pb]) & kKindBin) {
                     int c = (int)(ld_rlx32(&h->kind[ch * kChunkPages + pb]) & 0xFF);
                     bool empty = true;
-                    for (int i = 0; i < words_of(c); i++) if (w[i] & valid_mask(c, i)) empty = false;
+#pragma unroll
+                    for (int i = 0; i < 4; i++) if (i < words_of(c) && (w[i] & valid_mask(c, i))) empty = false;
                     if (empty) { pm_left |= 1ull << pb; }
                 }
             }
             if (budget > 0) budget--;
         }
         if (pm_left) {                                      // re-mark what could not go yet
-            if (a_or(&h->chunk_cand[ch], pm_left) == 0) hb3_set(cb, ch);
+            summarised_set(cb, ch, &h->chunk_cand[ch], pm_left);
             return;                                         // and stop: the rest is in use too
         }
     }
@@ -1003,7 +1032,7 @@ static __device__ __noinline__ uint64_t bin_claim_one(const ga_desc* h, uint32_t
         uint64_t ch = bin_find_chunk(h, A, c, &m);
         uint64_t p = ch * kChunkPages + (uint64_t)(__ffsll((long long)m) - 1);
         int wi;
-        uint64_t got = bin_claim_page(h, p, A, c, 1, &wi);
+        uint64_t got = bin_claim_page(h, p, A, c, 1, &wi, 0);
         if (got) return (p << kPageShift) + (uint64_t)(wi * 64 + __ffsll((long long)got) - 1) * csz;
     }
 }
@@ -1099,7 +1128,12 @@ static __device__ __noinline__ uint64_t bin_claim_collective(const ga_desc* h, u
     const uint32_t lane = lane_id();
     const uint32_t per_page = slots_of(c) < 64 ? slots_of(c) : 64;
     const uint64_t csz = 16ull << c;
+    // per-warp rotation of the page and word starts: the warps of an SM share
+    // the arena, so without it they all pile onto the first non-full page
+    uint32_t wid; asm volatile("mov.u32 %0, %%warpid;" : "=r"(wid));
+    const uint32_t rot = hash32(wid ^ (smid() << 6));
     uint64_t my = kNull;
+    uint32_t it = 0;                                        // retries move on to the next page
     unsigned unsat = grp;                                   // lanes still without a slot (this lane included)
     for (;;) {
         const int L = __ffs(unsat) - 1;
@@ -1109,12 +1143,12 @@ static __device__ __noinline__ uint64_t bin_claim_collective(const ga_desc* h, u
         m = __shfl_sync(unsat, m, L);
         const uint32_t q = __popc(unsat & lanemask_lt());
         const uint32_t np = __popcll(m);
-        const uint64_t page = ch * kChunkPages + nth_set(m, (q / per_page) % np);
+        const uint64_t page = ch * kChunkPages + nth_set(m, (q / per_page + rot + it++) % np);
         const unsigned pg = __match_any_sync(unsat, page);
         const int pl = __ffs(pg) - 1;
         uint64_t got = 0;
         int wi = 0;
-        if ((int)lane == pl) got = bin_claim_page(h, page, A, c, __popc(pg), &wi);
+        if ((int)lane == pl) got = bin_claim_page(h, page, A, c, __popc(pg), &wi, rot >> 8);
         got = __shfl_sync(pg, got, pl);
         wi = __shfl_sync(pg, wi, pl);
         const uint32_t pr = __popc(pg & lanemask_lt());
@@ -1398,7 +1432,8 @@ static __device__ __noinline__ void ga_free_off(const ga_desc* h, uint64_t off) 
             uint64_t ww[4];
             ld_bitmap(bw, ww);
             bool empty = true;
-            for (int i = 0; i < words_of(c); i++) if (ww[i] & valid_mask(c, i)) empty = false;
+#pragma unroll
+            for (int i = 0; i < 4; i++) if (i < words_of(c) && (ww[i] & valid_mask(c, i))) empty = false;
             if (empty) {
                 if (GA_SPAN_EAGER && is_span(c)) eager = true;   // reclaim after the signal below
                 else mark_candidate(h, p, A);
