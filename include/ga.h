@@ -98,6 +98,8 @@ typedef struct {
     uint64_t n_fallback;          /* group waits degraded to per-lane (R-27)               */
     uint64_t n_fail;              /* mallocs that returned NULL after every fallback       */
     uint64_t n_pending_reclaim;   /* candidate bins not yet reclaimed                      */
+    uint64_t n_repair_nonfull;    /* safety net: non-full bits re-published (expected 0)   */
+    uint64_t n_repair_summary;    /* safety net: chunk summary bits re-published (expected 0) */
     uint32_t n_arenas;
     uint32_t pad;
 } ga_stats_t;

@@ -45,7 +45,7 @@ class Stats(ctypes.Structure):
     _fields_ = [(n, ctypes.c_uint64) for n in (
         "heap_bytes", "metadata_bytes", "reserved_bytes", "peak_reserved_bytes", "n_bin_grow",
         "n_chunk_grow", "n_bin_reclaim", "n_chunk_reclaim", "n_fallback", "n_fail",
-        "n_pending_reclaim")] + [("n_arenas", ctypes.c_uint32), ("pad", ctypes.c_uint32)]
+        "n_pending_reclaim", "n_repair_nonfull", "n_repair_summary")] + [("n_arenas", ctypes.c_uint32), ("pad", ctypes.c_uint32)]
 
 
 class DevHeap(ctypes.Structure):

@@ -415,7 +415,6 @@ ga_status ga_l2_atomic_bench(ga_stream_t stream, int pattern, uint64_t* d_buf, u
 }
 
 ga_status ga_debug_attach(uint64_t** host_records) {
-#if GA_DEBUG
     if (!host_records) return GA_EINVAL;
     void* hp = nullptr;
     if (cudaHostAlloc(&hp, 8 * (8 + 4 * 256), cudaHostAllocMapped) != cudaSuccess) return GA_ENOMEM;
@@ -425,10 +424,6 @@ ga_status ga_debug_attach(uint64_t** host_records) {
     if (cudaMemcpyToSymbol(ga::g_ga_dbg, &dp, sizeof dp) != cudaSuccess) return GA_ECUDA;
     *host_records = (uint64_t*)hp;
     return GA_OK;
-#else
-    (void)host_records;
-    return GA_EINVAL;
-#endif
 }
 
 ga_status ga_bsem_bench(ga_stream_t stream, const ga_bsem_cfg* cfg, uint64_t* sems, uint64_t* out) {

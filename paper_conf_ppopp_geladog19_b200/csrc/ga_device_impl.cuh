@@ -85,10 +85,24 @@ constexpr int kMaxLevels = 48;
 #ifndef GA_MERGE_PRELOAD
 #define GA_MERGE_PRELOAD 1       // 1: try-wait loads the word before its fetch-add
 #endif
+#ifndef GA_INL_CLAIM
+#define GA_INL_CLAIM 1           // 1: inline the hint lookup and page claim into the collective claim
+#endif
+#ifndef GA_INL_WAIT
+#define GA_INL_WAIT 1            // 1: the arena-semaphore fast path inline at the malloc entry
+#endif
+#ifndef GA_FAST_FA
+#define GA_FAST_FA 1             // 1: that fast path is one fetch-add (no load gate)
+#endif
+#if GA_INL_CLAIM
+#define GA_CLAIM_FN __forceinline__
+#else
+#define GA_CLAIM_FN __noinline__
+#endif
 constexpr uint32_t kReclaimKeep = 64;           // free slots a delegated reclaim leaves per class
 
 enum { kStatBinGrow = 0, kStatChunkGrow, kStatBinReclaim, kStatChunkReclaim, kStatFallback,
-       kStatFail, kNumStats };
+       kStatFail, kStatRepairNonfull, kStatRepairSummary, kNumStats };
 
 static __device__ __forceinline__ uint32_t lane_id() { uint32_t r; asm volatile("mov.u32 %0, %%laneid;" : "=r"(r)); return r; }
 static __device__ __forceinline__ uint32_t lanemask_lt() { uint32_t r; asm volatile("mov.u32 %0, %%lanemask_lt;" : "=r"(r)); return r; }
@@ -142,8 +156,10 @@ static __device__ __forceinline__ void stat_add(const ga_desc* h, int i, uint64_
 #ifndef GA_DEBUG
 #define GA_DEBUG 0
 #endif
-#if GA_DEBUG
+// host-mapped diagnostics (ga_debug_attach); null unless attached.  Release
+// builds only touch it on the cold safety-net path (nfc_repair).
 static __device__ uint64_t* g_ga_dbg;
+#if GA_DEBUG
 #define SPIN_NOTE(cnt, site, a, b) spin_note((cnt), (site), (uint64_t)(a), (uint64_t)(b))
 #define GA_DBG_CNT uint32_t dbg_cnt = 0
 static __device__ __noinline__ void spin_note(uint32_t& cnt, int site, uint64_t a, uint64_t b) {
@@ -617,6 +633,10 @@ static __device__ __noinline__ void summarised_set(HB3 b, uint64_t ch, uint64_t*
     if ((ld_rlx(data) & bit) == bit && (ld_rlx(&b.w0[ch >> 6]) & cb)) return;
     if (a_or(data, bit) == 0 || !(ld_rlx(&b.w0[ch >> 6]) & cb)) hb3_set(b, ch);
 }
+static __device__ __forceinline__ void mark_candidate(const ga_desc* h, uint64_t p, uint32_t A) {
+    summarised_set(arena_hb(h, A, kAhbCnd), p >> kChunkShift, &h->chunk_cand[p >> kChunkShift],
+                   1ull << (p & (kChunkPages - 1)));
+}
 // page p (class c, arena A) has a free slot again
 static __device__ __forceinline__ void nonfull_set(const ga_desc* h, uint64_t p, int c, uint32_t A) {
     summarised_set(arena_hb(h, A, kAhbNfc + c), p >> kChunkShift, nonfull_word(h, p >> kChunkShift, c),
@@ -723,6 +743,15 @@ static __device__ __noinline__ void chunk_release(const ga_desc* h, uint64_t ch)
     if (A >= h->n_arenas) return;
     if (!bsem_trywait(psem_ptr(h, A), kChunkPages)) return;
     if (a_cas(&h->chunk_used[ch], 0ull, ~0ull) != 0ull) { bsem_signal(psem_ptr(h, A), kChunkPages, 0); return; }
+    // ABA (as in bin_reclaim): the chunk may have left A and come back empty
+    // under another arena between the owner read and the CAS.  It cannot move
+    // while its used word is all ones, so the owner read here decides.
+    if (const uint32_t o2 = ld_rlx32(&h->chunk_owner[ch]); o2 != A + 1) {
+        a_and(&h->chunk_used[ch], 0ull);
+        bsem_signal(psem_ptr(h, A), kChunkPages, 0);
+        if (o2 != 0) hb3_set(arena_hb(h, o2 - 1, kAhbFpc), ch);
+        return;
+    }
     hb3_clear_summarised(arena_hb(h, A, kAhbFpc), ch, &h->chunk_used[ch], ~0ull);
     if (a_exch(&h->chunk_cand[ch], 0)) hb3_clear_summarised(arena_hb(h, A, kAhbCnd), ch, &h->chunk_cand[ch], 0);
     st_rlx32(&h->chunk_owner[ch], 0);
@@ -758,7 +787,7 @@ static __device__ __forceinline__ void bin_init(const ga_desc* h, uint64_t p, ui
 // word scan starts at `rot` so concurrent warps on one page spread over its
 // words (scattered search).  Loops stay rolled: this is the hottest
 // code of the allocator and instruction-fetch stalls dominate.
-static __device__ __noinline__ uint64_t bin_claim_page(const ga_desc* h, uint64_t p, uint32_t A, int c, int need, int* wi,
+static __device__ GA_CLAIM_FN uint64_t bin_claim_page(const ga_desc* h, uint64_t p, uint32_t A, int c, int need, int* wi,
                                                        uint32_t rot) {
     uint64_t* bw = page_bits(h, p);
     uint64_t w[4];
@@ -840,10 +869,80 @@ static __device__ __noinline__ void nfc_audit(const ga_desc* h, uint32_t A, int 
 }
 #endif
 
+// Safety net for a claimer that holds units but finds no non-full (A, c) bin
+// for a long time (hundreds of microseconds: growers publish before they
+// signal, so a legitimate wait is short).  Walk arena A's chunks and re-publish
+// what the per-chunk words and summaries should show: (A, c) bins with a free
+// slot and no non-full bit, and non-full words whose chunk is missing from the
+// summary.  Each repair is counted (ga_stats n_repair_*), so a run that needed
+// one is visible; the measured runs of profiles/ report zero.
+static __device__ __noinline__ void nfc_repair(const ga_desc* h, uint32_t A, int c) {
+    HB3 nb = arena_hb(h, A, kAhbNfc + c);
+    const uint32_t step = is_span(c) ? kChunkPages : 1;
+    for (uint64_t ch = 0; ch < h->nchunks; ch++) {
+        if (ld_rlx32(&h->chunk_owner[ch]) != A + 1) continue;
+        uint64_t* nf = nonfull_word(h, ch, c);
+        for (uint32_t j = 0; j < kChunkPages; j += step) {
+            const uint64_t p = ch * kChunkPages + j;
+            if (ld_rlx32(&h->kind[p]) != kind_bin(A, c)) continue;
+            uint64_t w[4];
+            ld_bitmap(page_bits(h, p), w);
+            if (!page_full(w, c) && !((ld_rlx(nf) >> j) & 1)) {
+                summarised_set(nb, ch, nf, 1ull << j);
+                stat_add(h, kStatRepairNonfull, 1);
+            }
+        }
+        if (ld_rlx(nf) && !((ld_rlx(&nb.w0[ch >> 6]) >> (ch & 63)) & 1)) {
+            hb3_set(nb, ch);
+            stat_add(h, kStatRepairSummary, 1);
+        }
+    }
+    if (g_ga_dbg && atomicCAS((unsigned long long*)&g_ga_dbg[1], 0ull, 1ull) == 0ull) {
+        // one diagnostic dump (header words 2..7): where are arena A's class-c
+        // units?  Spans / bins of kind (A, c) anywhere, their free slots, how
+        // many sit in chunks not owned by A, how many lack their non-full bit.
+        uint64_t nb_all = 0, free_all = 0, foreign = 0, nf_missing = 0, free_foreign = 0;
+        for (uint64_t p = 0; p < h->pages; p += step) {
+            if (ld_rlx32(&h->kind[p]) != kind_bin(A, c)) continue;
+            uint64_t w[4];
+            ld_bitmap(page_bits(h, p), w);
+            uint64_t fr = 0;
+            for (int i = 0; i < 4; i++) if (i < words_of(c)) fr += __popcll(~w[i] & valid_mask(c, i));
+            nb_all++; free_all += fr;
+            const uint64_t ch = p >> kChunkShift;
+            if (ld_rlx32(&h->chunk_owner[ch]) != A + 1) { foreign++; free_foreign += fr; }
+            if (fr && !((ld_rlx(nonfull_word(h, ch, c)) >> (p & (kChunkPages - 1))) & 1)) nf_missing++;
+        }
+        // chunks owned by A + 1 and what their head page says
+        uint64_t owned = 0, owned_k0 = 0, owned_other = 0;
+        for (uint64_t ch = 0; ch < h->nchunks; ch++) {
+            if (ld_rlx32(&h->chunk_owner[ch]) != A + 1) continue;
+            owned++;
+            const uint32_t k = ld_rlx32(&h->kind[ch * kChunkPages]);
+            if (k == 0) owned_k0++;
+            else if (k != kind_bin(A, c)) owned_other++;
+        }
+        const uint64_t sw = ld_rlx(sem_ptr(h, A, c));
+        volatile uint64_t* r = (volatile uint64_t*)g_ga_dbg;
+        r[2] = ((uint64_t)A << 8) | (uint64_t)c | ((uint64_t)(uint32_t)sem_C(sw) << 32);
+        r[3] = nb_all; r[4] = free_all; r[5] = foreign | (free_foreign << 32); r[6] = nf_missing;
+        r[7] = ((uint64_t)(uint32_t)sem_D(sw) << 32);
+        r[8 + 4 * 255 + 0] = owned; r[8 + 4 * 255 + 1] = owned_k0; r[8 + 4 * 255 + 2] = owned_other;
+        r[8 + 4 * 255 + 3] = ld_rlx(&h->stats[kStatChunkGrow]) | (ld_rlx(&h->stats[kStatChunkReclaim]) << 32);
+        __threadfence_system();
+        r[1] = 2;
+    }
+    for (uint32_t j = 0; j < nb.n0; j++)                      // upper summary levels
+        if (ld_rlx(&nb.w0[j]) && !((ld_rlx(&hb3_w1(nb)[j >> 6]) >> (j & 63)) & 1)) {
+            hb3_up_set(nb, j);
+            stat_add(h, kStatRepairSummary, 1);
+        }
+}
+
 // A chunk of arena A with non-full class-c bins, and its non-full page mask:
 // the hint's chunk first, then the (A, c) summary.  Spins until one shows up
 // (the caller holds units, so a free slot exists or is being published).
-static __device__ __noinline__ uint64_t bin_find_chunk(const ga_desc* h, uint32_t A, int c, uint64_t* mask_out) {
+static __device__ GA_CLAIM_FN uint64_t bin_find_chunk(const ga_desc* h, uint32_t A, int c, uint64_t* mask_out) {
     GA_DBG_CNT;
     uint32_t hp = ld_rlx32(&h->hint[A * kNcls + c]);
     if (hp < h->pages) {                                      // the hint's chunk, if still A's
@@ -853,7 +952,7 @@ static __device__ __noinline__ uint64_t bin_find_chunk(const ga_desc* h, uint32_
     }
     HB3 nb = arena_hb(h, A, kAhbNfc + c);
     uint32_t seed = scatter_seed();
-    uint32_t ns = 32;
+    uint32_t ns = 32, spins = 0;
     for (;;) {
         int64_t j = hb3_find(nb, seed);
         if (j >= 0) {
@@ -878,6 +977,7 @@ static __device__ __noinline__ uint64_t bin_find_chunk(const ga_desc* h, uint32_
         SPIN_NOTE(dbg_cnt, 7, ((uint64_t)A << 8) | c, ns);
         __nanosleep(ns); if (ns < 1024) ns <<= 1;
         seed = hash32(seed + 7);
+        if ((++spins & 255) == 0) nfc_repair(h, A, c);
     }
 }
 
@@ -925,6 +1025,21 @@ static __device__ __noinline__ bool bin_reclaim(const ga_desc* h, uint64_t p, ui
         bsem_signal(sem_ptr(h, A, c), slots, 0);
         return false;
     }
+    // ABA: between the kind read and the CAS, p may have been reclaimed by
+    // someone else and re-made an empty bin of another arena (chunks move
+    // between arenas); the units just taken are then the wrong semaphore's.
+    // With every slot word now all ones the incarnation cannot change under
+    // us, so the kind read here decides: on a mismatch restore the words, give
+    // the units back and re-publish the page for its real owner.
+    if (const uint32_t k2 = ld_rlx32(&h->kind[p]); k2 != k) {
+        for (int q = 0; q < words_of(c); q++) a_and(&bw[q], ~valid_mask(c, q));
+        bsem_signal(sem_ptr(h, A, c), slots, 0);
+        if ((k2 & 0xC0000000u) == kKindBin) {
+            nonfull_set(h, p, (int)(k2 & 0xFF), (k2 >> 8) & 0xFFFFu);
+            mark_candidate(h, p, (k2 >> 8) & 0xFFFFu);
+        }
+        return false;
+    }
     uint64_t ch = p >> kChunkShift;
     uint64_t* nf = nonfull_word(h, ch, c);
     uint64_t bit = 1ull << (p & (kChunkPages - 1));
@@ -937,10 +1052,6 @@ static __device__ __noinline__ bool bin_reclaim(const ga_desc* h, uint64_t p, ui
     return true;
 }
 
-static __device__ __forceinline__ void mark_candidate(const ga_desc* h, uint64_t p, uint32_t A) {
-    summarised_set(arena_hb(h, A, kAhbCnd), p >> kChunkShift, &h->chunk_cand[p >> kChunkShift],
-                   1ull << (p & (kChunkPages - 1)));
-}
 
 // Reclaim up to `budget` candidate bins of arena A (budget < 0: all), leaving
 // at least `keep` free slots per class (0: reclaim every empty bin).
@@ -1135,7 +1246,9 @@ static __device__ __noinline__ uint64_t bin_claim_collective(const ga_desc* h, u
     uint64_t my = kNull;
     uint32_t it = 0;                                        // retries move on to the next page
     unsigned unsat = grp;                                   // lanes still without a slot (this lane included)
+    GA_DBG_CNT;
     for (;;) {
+        SPIN_NOTE(dbg_cnt, 10, ((uint64_t)A << 8) | c, unsat);
         const int L = __ffs(unsat) - 1;
         uint64_t ch = 0, m = 0;
         if ((int)lane == L) ch = bin_find_chunk(h, A, c, &m);
@@ -1355,7 +1468,25 @@ static __device__ __noinline__ uint64_t ga_malloc_off(const ga_desc* h, uint64_t
         const int leader = __ffs(grp) - 1;
         int r = 0;
         if ((int)lane_id() == leader)
-            r = bsem_wait(sem_ptr(h, A, key), N, slots * ((N + slots - 1) / slots), ArenaSpin{h, A});
+        {
+            uint64_t* sp = sem_ptr(h, A, key);
+#if GA_INL_WAIT
+            // inline fast path: the units are there -> one fetch-add decides
+            const uint64_t dn = (uint64_t)N << 32;
+            r = kBlocked;
+#if GA_FAST_FA
+            {
+#else
+            if (sem_C(ld_rlx(sp)) >= (int32_t)N) {
+#endif
+                uint64_t old = a_add(sp, (uint64_t)0 - dn);
+                if (sem_C(old) >= (int32_t)N) r = kAcquired;
+                else a_add(sp, dn);
+            }
+            if (r != kAcquired)
+#endif
+            r = bsem_wait(sp, N, slots * ((N + slots - 1) / slots), ArenaSpin{h, A});
+        }
         r = __shfl_sync(grp, r, leader);
         my = r == kAcquired ? bin_claim_collective(h, grp, A, key)
            : is_span(key) ? span_grow_collective(h, grp, A, key) : bin_grow_collective(h, grp, A, key);

@@ -300,6 +300,8 @@ ga_status ga_stats(ga_heap_t h, ga_stream_t stream, ga_stats_t* out) {
     out->n_fallback = st[kStatFallback];
     out->n_fail = st[kStatFail];
     out->n_pending_reclaim = pend;
+    out->n_repair_nonfull = st[kStatRepairNonfull];
+    out->n_repair_summary = st[kStatRepairSummary];
     out->n_arenas = h->dev.n_arenas;
     return GA_OK;
 }

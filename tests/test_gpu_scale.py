@@ -66,6 +66,44 @@ def test_d4_full_grid_pressure_valid():
     _empty(heap)
 
 
+def test_d4_full_grid_exhaust_valid():
+    """d4 exhaust level (3 GiB heap, ~95 % live after rounding): mallocs fail and
+    deferred reclamation runs under near-exhaustion.  The log still passes the
+    oracle checker (failed calls are NULL records), frees are exact, the heap is
+    empty after quiesce, and failures stay within a small fraction of the calls
+    (the oracle's own count is the reference point, not an exact target: the
+    two place blocks differently under pressure)."""
+    t = tracegen.d4_mixed("exhaust", R=6)
+    ref = oracle.run_trace(t.sizes, t.heap_bytes, t.D, want_ok=False)
+    heap = GpuHeap(t.heap_bytes)
+    run = run_correctness(heap, t.sizes, t.D)
+    err, cs = oracle.check_log(run.log, t.R, t.T, t.D, t.heap_bytes)
+    assert err == 0, (err, cs)
+    assert run.counts["tag_errors"] == 0
+    assert run.counts["n_malloc"] == ref.stats["n_malloc"]
+    assert run.counts["n_free"] == run.counts["n_malloc"] - run.counts["n_fail"]
+    assert run.counts["n_fail"] <= max(4 * ref.stats["n_malloc_fail"], run.counts["n_malloc"] // 50), \
+        (run.counts, ref.stats["n_malloc_fail"])
+    _empty(heap)
+
+
+@pytest.mark.timeout(600, method="thread")
+@pytest.mark.parametrize("size", [16, 256, 4096])
+def test_timed_kernel_liveness_repeated(size):
+    """The timed kernel finishes, rep after rep, on warp-uniform bin and span
+    classes (a lost non-full summary once hung span arenas after ~100 reps)."""
+    t = tracegen.d3_uniform(size, R=16)
+    heap = GpuHeap(t.heap_bytes)
+    d = torch.from_numpy(t.sizes.view(np.int32)).cuda()
+    c = torch.zeros(8, dtype=torch.int64, device="cuda")
+    for _ in range(60):
+        run_timed(heap, d, t.R, t.T, t.D, c)
+    torch.cuda.synchronize()
+    cc = c.cpu().numpy()
+    assert cc[0] == cc[2] == 60 * t.R * t.T and cc[1] == 0
+    _empty(heap)
+
+
 @pytest.mark.parametrize("size", [16, 2048, 8192])
 def test_d3_full_grid_correctness(size):
     t = tracegen.d3_uniform(size, R=2)
@@ -141,13 +179,15 @@ def test_l2_atomic_bench_plausible():
     s = torch.cuda.current_stream()
     rates = {}
     for pat in range(6):
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         iters = 16 if pat < 4 else 4
-        e0.record(s)
-        ga.ga_l2_atomic_bench(s.cuda_stream, pat, buf.data_ptr(), buf.numel(), iters, 148 * 8, 256, sink.data_ptr())
-        e1.record(s)
-        e1.synchronize()
-        rates[pat] = 148 * 8 * 256 * iters / (e0.elapsed_time(e1) / 1e3)
+        for rep in range(3):                            # the first launch is cold (module load)
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(s)
+            ga.ga_l2_atomic_bench(s.cuda_stream, pat, buf.data_ptr(), buf.numel(), iters, 148 * 8, 256,
+                                  sink.data_ptr())
+            e1.record(s)
+            e1.synchronize()
+            rates[pat] = max(rates.get(pat, 0.0), 148 * 8 * 256 * iters / (e0.elapsed_time(e1) / 1e3))
     assert rates[1] > 1e10 and rates[0] > 1e10         # distinct-word atomics: > 10 Gatom/s
     assert rates[2] < rates[0]                          # one hot word is slower than spread words
     assert int(buf[0].item()) > 0

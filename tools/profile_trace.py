@@ -18,6 +18,7 @@ ap.add_argument("--reps", type=int, default=3)
 ap.add_argument("--cuda", action="store_true")
 ap.add_argument("--kmin", type=int, default=3)
 ap.add_argument("--kmax", type=int, default=15)
+ap.add_argument("--threads", type=int, default=0, help="fewer threads than the full grid (sanitizer runs)")
 a = ap.parse_args()
 if a.workload == "d4":
     t = tracegen.d4_mixed("pressure", R=a.rounds)
@@ -25,6 +26,8 @@ if a.workload == "d4":
         t = tracegen.Trace("d4_sub", tracegen.mixed_sizes(t.seed, a.rounds, t.T, a.kmin, a.kmax), 1, t.heap_bytes, t.seed)
 else:
     t = tracegen.d3_uniform(a.size, R=a.rounds)
+if a.threads:
+    t = tracegen.Trace(t.name, np.ascontiguousarray(t.sizes[:, :a.threads]), t.D, t.heap_bytes, t.seed)
 torch.cuda.set_device(0)
 heap = None if a.cuda else GpuHeap(t.heap_bytes)
 if a.cuda:
@@ -39,3 +42,6 @@ for i in range(a.reps):
     e.record()
     e.synchronize()
     print(f"rep {i}: {s.elapsed_time(e):.2f} ms, counts {c.cpu().numpy()[:4]}", flush=True)
+if heap is not None:
+    st = heap.stats()
+    print("stats", {k: st[k] for k in ("n_repair_nonfull", "n_repair_summary", "n_fallback", "n_fail")}, flush=True)
