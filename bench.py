@@ -217,10 +217,12 @@ def d3_sweep(ga, heap, stream, dev, T, args, sizes=(16, 32, 64, 128, 256, 512, 1
     return res
 
 
-def d4_levels(ga, stream, dev, args, flush, levels=("fit", "exhaust"), reps=3):
+def d4_levels(ga, stream, dev, args, flush, levels=("fit", "exhaust", "overcommit"), reps=3):
     """d4 at the other two pressure levels: the same mixed trace on
-    a 16 GiB heap (fit: every malloc succeeds) and a 3 GiB heap (exhaust: ~95 %
-    rounded-live, failures and deferred reclamation).  calls/s from the timed
+    a 16 GiB heap (fit: every malloc succeeds), a 3 GiB heap (exhaust: the peak
+    reserved reaches ~99 % of the heap) and a 2.75 GiB heap (overcommit: below
+    the oracle's own peak reserved, so both sides fail mallocs and reclaim under
+    real exhaustion).  calls/s from the timed
     kernel; failures and fragmentation from correctness mode, beside the oracle's."""
     import torch
     import oracle
@@ -252,7 +254,7 @@ def d4_levels(ga, stream, dev, args, flush, levels=("fit", "exhaust"), reps=3):
         fo = ref["peak_reserved_bytes"] / ref["peak_live_bytes"]
         st = heap.stats()
         res[lv] = {"heap_bytes": t.heap_bytes, "calls_per_s": calls / (sum(times) / len(times)),
-                   "ms": sum(times) / len(times), "timed_failed_mallocs": fails,
+                   "ms": 1e3 * sum(times) / len(times), "timed_failed_mallocs": fails,
                    "correctness_failed_mallocs": run.counts["n_fail"], "oracle_failed_mallocs": ref["n_malloc_fail"],
                    "fragmentation": {"gpu": fg, "oracle": fo, "ratio": fg / fo if fg else None},
                    "stats": {k: int(v) for k, v in st.items() if isinstance(v, (int, np.integer))}}

@@ -225,9 +225,12 @@ __global__ void k_bsem(ga_bsem_cfg cfg, uint64_t* sems, uint64_t* out, uint32_t 
                 if (!cfg.acquire_only) ga_bsem_signal((ga_bsem*)s, N, 0);
             }
             __syncwarp(act);
-        } else if (cfg.variant == 1) {
+        } else if (cfg.variant == 1 || cfg.variant == 4) {
+            // 1: exact form (CAS decisions); 4: fetch-add form (every update one
+            // fetch-add, as the paper's R-saturation note implies)
             uint32_t Bp = cfg.B * ((k + cfg.B - 1) / cfg.B);
-            int r = ga_bsem_wait((ga_bsem*)s, k, Bp);
+            int r = cfg.variant == 1 ? ga_bsem_wait((ga_bsem*)s, k, Bp)
+                                     : ga::bsem_wait_fast((uint64_t*)s, k, Bp, ga::NoSpin());
             waits++;
             if (r == GA_GROW) {
                 atomicAdd((unsigned long long*)bump + (tid & zero), (unsigned long long)Bp);
@@ -278,7 +281,7 @@ __global__ void k_bsem_final(uint32_t n_sems, const uint64_t* sems, uint64_t* ou
     for (uint32_t i = 0; i < n_sems; i++) {
         uint64_t w = sems[i * 4];
         int64_t C, D;
-        if (variant <= 1) { C = (int32_t)(uint32_t)(w >> 32); D = (int32_t)((uint32_t)w - 0x80000000u); }
+        if (variant <= 1 || variant == 4) { C = (int32_t)(uint32_t)(w >> 32); D = (int32_t)((uint32_t)w - 0x80000000u); }
         else if (variant == 2) { C = (int32_t)(uint32_t)w; D = 0; }
         else { C = (int64_t)w; D = 0; }
         sc += C;
@@ -288,7 +291,7 @@ __global__ void k_bsem_final(uint32_t n_sems, const uint64_t* sems, uint64_t* ou
 }
 __global__ void k_bsem_init(uint32_t n_sems, uint64_t* sems, uint32_t variant) {
     uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
-    if (i < n_sems * 4 + 4) sems[i] = (variant <= 1 && i < n_sems * 4) ? 0x80000000ull : 0ull;
+    if (i < n_sems * 4 + 4) sems[i] = ((variant <= 1 || variant == 4) && i < n_sems * 4) ? 0x80000000ull : 0ull;
 }
 
 // resident 256-thread blocks per SM the timed kernel is compiled for (register
@@ -427,7 +430,7 @@ ga_status ga_debug_attach(uint64_t** host_records) {
 }
 
 ga_status ga_bsem_bench(ga_stream_t stream, const ga_bsem_cfg* cfg, uint64_t* sems, uint64_t* out) {
-    if (!cfg || !sems || !out || cfg->variant > 3 || cfg->B == 0 || cfg->n_sems == 0 || cfg->k > 32) return GA_EINVAL;
+    if (!cfg || !sems || !out || cfg->variant > 4 || cfg->B == 0 || cfg->n_sems == 0 || cfg->k > 32) return GA_EINVAL;
     cudaStream_t s = (cudaStream_t)stream;
     k_bsem_init<<<(cfg->n_sems * 4 + 4 + 255) / 256, 256, 0, s>>>(cfg->n_sems, sems, cfg->variant);
     cudaMemsetAsync(out, 0, 64, s);

@@ -94,6 +94,9 @@ constexpr int kMaxLevels = 48;
 #ifndef GA_FAST_FA
 #define GA_FAST_FA 1             // 1: that fast path is one fetch-add (no load gate)
 #endif
+#ifndef GA_HINT_LDCA
+#define GA_HINT_LDCA 0           // 1: read the per-(arena, class) hint through L1
+#endif
 #if GA_INL_CLAIM
 #define GA_CLAIM_FN __forceinline__
 #else
@@ -944,7 +947,13 @@ static __device__ __noinline__ void nfc_repair(const ga_desc* h, uint32_t A, int
 // (the caller holds units, so a free slot exists or is being published).
 static __device__ GA_CLAIM_FN uint64_t bin_find_chunk(const ga_desc* h, uint32_t A, int c, uint64_t* mask_out) {
     GA_DBG_CNT;
+#if GA_HINT_LDCA
+    // the hint is only a hint: an L1-cached (possibly stale) read saves an L2
+    // round trip; the chunk's owner and non-full word below are read fresh
+    uint32_t hp = __ldca(&h->hint[A * kNcls + c]);
+#else
     uint32_t hp = ld_rlx32(&h->hint[A * kNcls + c]);
+#endif
     if (hp < h->pages) {                                      // the hint's chunk, if still A's
         const uint32_t own = ld_rlx32(&h->chunk_owner[hp >> kChunkShift]);
         uint64_t m = ld_rlx(nonfull_word(h, hp >> kChunkShift, c));

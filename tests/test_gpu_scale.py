@@ -87,6 +87,24 @@ def test_d4_full_grid_exhaust_valid():
     _empty(heap)
 
 
+def test_d4_full_grid_overcommit_valid():
+    """d4 on a 2.75 GiB heap, below the oracle's own peak reserved: both sides
+    fail mallocs.  The log passes the checker, the heap empties after quiesce,
+    and the GPU's failures stay within a small multiple of the oracle's (they
+    place blocks differently, so counts are not compared exactly, R-26)."""
+    t = tracegen.d4_mixed("overcommit", R=8)
+    ref = oracle.run_trace(t.sizes, t.heap_bytes, t.D, want_ok=False)
+    heap = GpuHeap(t.heap_bytes)
+    run = run_correctness(heap, t.sizes, t.D)
+    err, cs = oracle.check_log(run.log, t.R, t.T, t.D, t.heap_bytes)
+    assert err == 0, (err, cs)
+    assert run.counts["tag_errors"] == 0
+    assert run.counts["n_free"] == run.counts["n_malloc"] - run.counts["n_fail"]
+    assert run.counts["n_fail"] <= 3 * ref.stats["n_malloc_fail"] + run.counts["n_malloc"] // 100, \
+        (run.counts, ref.stats["n_malloc_fail"])
+    _empty(heap)
+
+
 @pytest.mark.timeout(600, method="thread")
 @pytest.mark.parametrize("size", [16, 256, 4096])
 def test_timed_kernel_liveness_repeated(size):

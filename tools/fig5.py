@@ -7,7 +7,10 @@ batch with one atomic on a bump counter.  One semaphore for the
 whole grid, as in the paper.  Swept over the number of concurrent threads
 (multiple waves above the 303,104 resident threads), for
   counting  -- the growable counting semaphore of Sec. 3.2,
-  bulk      -- Alg. 1 / Alg. 2 per thread (the paper's bulk semaphore),
+  bulk      -- Alg. 1 / Alg. 2 per thread, exact form (one CAS decides each wait),
+  bulk_fa   -- Alg. 1 / Alg. 2 per thread, fetch-add form (each update one
+               fetch-add: the paper's "updates to R saturate the atomic
+               throughput", P:L1384-1402),
   bulk_warp -- Alg. 1 / Alg. 2 with one wait per warp for the warp's N units
                (this build's warp aggregation, subsystem 1 of the north star).
 Each point checks the acquire-only invariant of pin P-2: batches produced =
@@ -28,7 +31,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 
 THREADS = [1024, 4096, 16384, 65536, 131072, 262144, 303104, 393216, 524288, 606208]
-NAMES = {2: "counting", 1: "bulk", 0: "bulk_warp"}
+NAMES = {2: "counting", 1: "bulk", 4: "bulk_fa", 0: "bulk_warp"}
 
 
 def main():
@@ -47,7 +50,7 @@ def main():
     rows = []
     for T in THREADS:
         row = {"threads": T}
-        for v in (2, 1, 0):
+        for v in (2, 1, 4, 0):
             per_block = {}
             for blk in blocks:
                 grid = (T + blk - 1) // blk
@@ -74,7 +77,7 @@ def main():
         rows.append(row)
         print(f"T={T:>7d}  " + "  ".join(f"{NAMES[v]} {row[NAMES[v]]['allocs_per_s_block256']:.3e}/s"
                                          f"{'' if row[NAMES[v]]['invariants_ok'] else ' (INVARIANT FAIL)'}"
-                                         for v in (2, 1, 0)), flush=True)
+                                         for v in (2, 1, 4, 0)), flush=True)
     res = {"experiment": "Fig. 5 (P:L1324-1402): acquire-only, one unit per thread, B = %d, one semaphore" % a.B,
            "blocks": blocks, "rows": rows}
     if a.out:

@@ -103,7 +103,9 @@ def mixed_sizes(seed: int, R: int, T: int, kmin: int = 3, kmax: int = 15) -> np.
 
 
 def d4_mixed(level: str = "pressure", T: int = FULL_GRID_THREADS, R: int = 16) -> Trace:
-    heap = {"fit": 16 << 30, "pressure": 4 << 30, "exhaust": 3 << 30}[level]
+    # overcommit: 2.75 GiB, below the oracle's own peak reserved (3.07 GB), so
+    # both sides fail some mallocs and reclaim under real exhaustion
+    heap = {"fit": 16 << 30, "pressure": 4 << 30, "exhaust": 3 << 30, "overcommit": 11 << 28}[level]
     seed = BASE_SEED + 4
     return Trace(f"d4_mixed_{level}", mixed_sizes(seed, R, T), 1, heap, seed)
 
