@@ -141,11 +141,7 @@ ga_status ga_heap_create(int device, ga_stream_t stream, void* buf, size_t bytes
     d.L = L;
     int nsm = 0;
     cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, device);
-    // One arena per SM, but at least kMinArenaChunks chunks per arena:
-    // a small pool split 148 ways leaves most arenas without a chunk, and their
-    // mallocs then live on the cross-arena fallback (Fig. 7's 8-16 MB pools).
-    d.n_arenas = nsm > 0 ? (uint32_t)nsm : 1;
-    if (d.n_arenas > nchunks / kMinArenaChunks) d.n_arenas = nchunks / kMinArenaChunks > 0 ? (uint32_t)(nchunks / kMinArenaChunks) : 1;
+    d.n_arenas = nsm > 0 ? (uint32_t)nsm : 1;             // one arena per SM
     d.chunk_words = (uint32_t)((nchunks + 63) / 64);
     d.flags = flags;
     // tree levels

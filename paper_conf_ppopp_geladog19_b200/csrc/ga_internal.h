@@ -6,8 +6,6 @@
 
 #include "ga.h"
 
-constexpr uint64_t kMinArenaChunks = 8;   // fewer arenas than SMs below 8 chunks per arena
-
 struct ga_heap_s {
     int device = 0;
     char* pool_raw = nullptr;      // owned pool allocation (nullptr if borrowed)
