@@ -424,8 +424,12 @@ def main():
     a_min = algorithmic_atomics(trace.sizes)
     achieved = a_min / (ms / 1e3) / 1e9
     kinfo = ga.ga_kernel_info(0, args.block)
+    traffic = None                                          # DRAM bytes per launch, from the committed ncu capture
+    tf = os.path.join(ROOT, "profiles", "r01_ncu_traffic.json")
+    if os.path.exists(tf):
+        traffic = json.load(open(tf)).get("traffic_bytes")
     roofline = {"bound": "l2_atomic", "achieved": achieved, "peak": p_atom, "unit": "Gatom/s",
-                "frac": achieved / p_atom, "traffic": None,
+                "frac": achieved / p_atom, "traffic": traffic, "traffic_unit": "DRAM bytes per launch (ncu)",
                 "per_launch_algorithmic_atomics": a_min,
                 "peak_source": "measured live: ga_l2_atomic_bench distinct-word ATOMG/REDG (max)",
                 "peak_patterns_gatom_s": {"atomg_distinct": peaks[0], "redg_distinct": peaks[1],

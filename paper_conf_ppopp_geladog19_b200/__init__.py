@@ -18,7 +18,8 @@ __all__ = ["lib", "GaError", "Layout", "Stats", "DevHeap", "ga_heap_create", "ga
            "ga_heap_quiesce", "ga_heap_snapshot", "ga_reserved_pages", "ga_status_str",
            "ga_trace_phase", "ga_trace_timed", "ga_trace_timed_host", "ga_cuda_set_heap_limit",
            "ga_cuda_trace_phase", "ga_cuda_trace_timed", "ga_kernel_info", "ga_l2_atomic_bench",
-           "ga_bsem_bench", "BsemCfg", "EXPORTED", "GA_TRACE_LOG", "GA_TRACE_TAG"]
+           "ga_bsem_bench", "BsemCfg", "EXPORTED", "GA_TRACE_LOG", "GA_TRACE_TAG",
+           "ga_rcu_workspace_bytes", "ga_rcu_list_removal"]
 
 GA_TRACE_LOG = 1
 GA_TRACE_TAG = 2
@@ -28,7 +29,8 @@ EXPORTED = ["ga_heap_create", "ga_heap_destroy", "ga_heap_reset", "ga_stats", "g
             "ga_heap_info", "ga_layout", "ga_heap_quiesce", "ga_heap_snapshot", "ga_reserved_pages",
             "ga_status_str", "ga_trace_phase", "ga_trace_timed", "ga_trace_timed_host",
             "ga_cuda_set_heap_limit", "ga_cuda_trace_phase", "ga_cuda_trace_timed",
-            "ga_kernel_info", "ga_l2_atomic_bench", "ga_bsem_bench", "ga_debug_attach"]
+            "ga_kernel_info", "ga_l2_atomic_bench", "ga_bsem_bench", "ga_debug_attach",
+            "ga_rcu_workspace_bytes", "ga_rcu_list_removal"]
 
 
 class GaError(RuntimeError):
@@ -96,6 +98,8 @@ def lib():
         "ga_l2_atomic_bench": [vp, i32, vp, u64, u32, u32, u32, vp],
         "ga_bsem_bench": [vp, P(BsemCfg), vp, vp],
         "ga_debug_attach": [P(P(u64))],
+        "ga_rcu_workspace_bytes": [u32, P(sz)],
+        "ga_rcu_list_removal": [vp, u32, u32, vp, vp, sz, u32, u32, vp],
     }
     for name, args in sig.items():
         f = getattr(L, name)
@@ -210,6 +214,17 @@ def ga_kernel_info(which: int, block: int = 256) -> dict:
 def ga_l2_atomic_bench(stream, pattern, buf, n_words, iters, grid, block, sink):
     _ok(lib().ga_l2_atomic_bench(stream or None, pattern, buf, n_words, iters, grid, block, sink),
         "ga_l2_atomic_bench")
+
+
+def ga_rcu_workspace_bytes(n_nodes: int) -> int:
+    out = ctypes.c_size_t()
+    _ok(lib().ga_rcu_workspace_bytes(n_nodes, ctypes.byref(out)), "ga_rcu_workspace_bytes")
+    return out.value
+
+
+def ga_rcu_list_removal(stream, n_threads, n_nodes, tags, ws, ws_bytes, delegate, block, out):
+    _ok(lib().ga_rcu_list_removal(stream or None, n_threads, n_nodes, tags, ws, ws_bytes, delegate, block, out),
+        "ga_rcu_list_removal")
 
 
 def ga_bsem_bench(stream, cfg: BsemCfg, sems, out):

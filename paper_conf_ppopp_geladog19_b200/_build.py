@@ -14,9 +14,9 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
 LIB = os.path.join(PKG, "libga.so")
-SOURCES = ["ga_host.cu", "ga_bench.cu"]
+SOURCES = ["ga_host.cu", "ga_bench.cu", "ga_rcu.cu"]
 DEPS = SOURCES + ["ga_device_impl.cuh", "ga_internal.h"]
-HEADERS = ["ga.h", "ga_bench.h", "ga_device.cuh"]
+HEADERS = ["ga.h", "ga_bench.h", "ga_device.cuh", "ga_rcu.h"]
 
 NVCC_FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo", "-O3", "-std=c++17",
               "-Xcompiler", "-fPIC", "-shared", "-Xptxas", "-warn-spills"]

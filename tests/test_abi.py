@@ -14,7 +14,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 def _declared():
     names = set()
-    for h in ("ga.h", "ga_bench.h"):
+    for h in ("ga.h", "ga_bench.h", "ga_rcu.h"):
         src = open(os.path.join(ROOT, "include", h)).read()
         names |= set(re.findall(r"^\s*(?:ga_status|const char\*)\s+(ga_\w+)\s*\(", src, re.M))
     return names

@@ -113,3 +113,13 @@ def d4_mixed(level: str = "pressure", T: int = FULL_GRID_THREADS, R: int = 16) -
 def d4_small(T: int = 4096, R: int = 8, heap_bytes: int = 64 << 20, seed: int = BASE_SEED + 40) -> Trace:
     """Reduced mixed trace for parity tests the oracle finishes in well under a second."""
     return Trace("d4_small", mixed_sizes(seed, R, T), 1, heap_bytes, seed)
+
+
+def rcu_tags(T: int, W: int, seed: int = BASE_SEED + 6) -> np.ndarray:
+    """Fig. 6 input: the W list tags 0..W-1 once each (writers)
+    and T - W tags >= W that are not in the list (readers), in a seeded random
+    order (splitmix64 keys, argsort)."""
+    assert 0 < W <= T
+    tags = np.concatenate([np.arange(W, dtype=np.uint32), W + np.arange(T - W, dtype=np.uint32)])
+    keys = splitmix64(np.uint64(seed) ^ (np.arange(T, dtype=np.uint64) * np.uint64(0x9E3779B97F4A7C15)))
+    return tags[np.argsort(keys, kind="stable")]
