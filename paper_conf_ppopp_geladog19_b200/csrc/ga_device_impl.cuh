@@ -60,10 +60,10 @@ constexpr int kNcls = kNbin + kNspan;           // classes 0 .. kNcls-1
 // "Spans").  GA_SPAN_EAGER=1: a free that empties a span returns it to the
 // tree at once when the class keeps a span's worth of free slots elsewhere.
 #ifndef GA_SPAN_SHARE
-#define GA_SPAN_SHARE 4
+#define GA_SPAN_SHARE 2
 #endif
 #ifndef GA_SPAN_EAGER
-#define GA_SPAN_EAGER 1
+#define GA_SPAN_EAGER 0
 #endif
 constexpr int kMinShift = 4;                    // 16 B minimum class (R-13)
 constexpr int kBinWords = 4;                    // 256-bit slot bitmap per page

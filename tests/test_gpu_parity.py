@@ -100,6 +100,38 @@ def test_single_class_exhaust_exact(size):
     _empty_parity(heap)
 
 
+@pytest.mark.parametrize("size", [65536, 131072, 524288, 2 << 20])
+def test_single_class_exhaust_exact_tree_sizes(size):
+    """The same for spans' largest class and TBuddy orders above it (Fig. 7's
+    64 KiB - 512 KiB points and beyond): counts equal capacity exactly."""
+    heap_bytes = 64 << 20
+    cap = heap_bytes // size
+    sizes = np.full((1, cap + 32), size, dtype=np.uint32)
+    ref = oracle.run_trace(sizes, heap_bytes, 0)
+    assert ref.stats["n_malloc_fail"] == 32
+    heap = GpuHeap(heap_bytes)
+    run = run_correctness(heap, sizes, 0)
+    assert run.counts["n_malloc"] - run.counts["n_fail"] == cap
+    _check_log(run, sizes, 0, heap_bytes)
+    _empty_parity(heap)
+
+
+def test_mixed_churn_up_to_1mib():
+    """Mixed churn with classes 16 B - 1 MiB (octaves 3..19): bins, spans and
+    TBuddy orders 5-8 in one warp; fit-level heap, so counts equal the
+    oracle's; the log passes and the heap empties."""
+    T, R = 4096, 6
+    sizes = tracegen.mixed_sizes(tracegen.BASE_SEED + 41, R, T, 3, 19)
+    heap_bytes = 4 << 30
+    ref = oracle.run_trace(sizes, heap_bytes, 1)
+    assert ref.stats["n_malloc_fail"] == 0
+    heap = GpuHeap(heap_bytes)
+    run = run_correctness(heap, sizes, 1)
+    assert run.counts["n_fail"] == 0 and run.counts["n_malloc"] == ref.stats["n_malloc"]
+    _check_log(run, sizes, 1, heap_bytes)
+    _empty_parity(heap)
+
+
 def test_d4_small_fit_churn():
     """config d4 (reduced, fit): mixed 16 B - 64 KiB churn, D = 1; counts equal."""
     t = tracegen.d4_small(T=8192, R=8, heap_bytes=256 << 20)
