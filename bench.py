@@ -293,6 +293,27 @@ def d2_bsem(ga, stream, dev, grid=148 * 8, block=256, iters=32):
     return res
 
 
+# ----------------------------------------------------------------------------- multi-GPU (replicas)
+def rank_trace(trace, rank: int):
+    """Replicas (DESIGN.md section 8): rank r runs the same recipe with seed + r;
+    rank 0 runs the canonical bench trace."""
+    if rank == 0:
+        return trace
+    return tracegen.Trace(trace.name, tracegen.mixed_sizes(trace.seed + rank, trace.R, trace.T), trace.D,
+                          trace.heap_bytes, trace.seed + rank)
+
+
+def reduce_over_ranks(dist, ms: float, calls: float, device):
+    """Whole-job numbers: the slowest rank's time and the calls of all ranks."""
+    import torch
+    t = torch.tensor([ms], device=device, dtype=torch.float64)
+    c = torch.tensor([calls], device=device, dtype=torch.float64)
+    if dist is not None:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        dist.all_reduce(c, op=dist.ReduceOp.SUM)
+    return float(t.item()), float(c.item())
+
+
 # ----------------------------------------------------------------------------- our arm
 def main():
     ap = argparse.ArgumentParser()
@@ -326,9 +347,7 @@ def main():
     stream = torch.cuda.current_stream(dev)
 
     # per-rank trace (replicas: seed + rank); rank 0 uses the canonical trace
-    if rank:
-        trace = tracegen.Trace(trace.name, tracegen.mixed_sizes(trace.seed + rank, trace.R, trace.T), trace.D,
-                               trace.heap_bytes, trace.seed + rank)
+    trace = rank_trace(trace, rank)
     R, T, D = trace.R, trace.T, trace.D
     if not args.no_extras:
         ga.ga_cuda_set_heap_limit(trace.heap_bytes)       # before any kernel that uses malloc
@@ -366,13 +385,8 @@ def main():
     c = counts.cpu().numpy()
     calls_step = int(c[0] + c[2]) // args.steps
     fails_step = int(c[1]) // args.steps
-    t_max = torch.tensor([ms], device=dev, dtype=torch.float64)
-    tot_calls = torch.tensor([calls_step], device=dev, dtype=torch.float64)
-    if dist:
-        dist.all_reduce(t_max, op=dist.ReduceOp.MAX)
-        dist.all_reduce(tot_calls, op=dist.ReduceOp.SUM)
-    ms_max = float(t_max.item())
-    value = float(tot_calls.item()) / (ms_max / 1e3)
+    ms_max, tot = reduce_over_ranks(dist, ms, calls_step, dev)
+    value = tot / (ms_max / 1e3)
 
     # ---- e2e: host buffers through the C ABI (H2D of the trace, kernel, D2H of counts)
     h_sizes = torch.from_numpy(trace.sizes.view(np.int32)).pin_memory()
@@ -389,14 +403,10 @@ def main():
         if i >= args.warmup:
             e2e_ms.append(s0.elapsed_time(s1))
     e2e_calls = int(h_counts[0] + h_counts[2])
-    e2e_t = torch.tensor([sum(e2e_ms) / len(e2e_ms)], device=dev, dtype=torch.float64)
-    e2e_c = torch.tensor([e2e_calls], device=dev, dtype=torch.float64)
-    if dist:
-        dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
-        dist.all_reduce(e2e_c, op=dist.ReduceOp.SUM)
-    e2e = {"value": float(e2e_c.item()) / (float(e2e_t.item()) / 1e3), "unit": UNIT,
+    e2e_ms_max, e2e_tot = reduce_over_ranks(dist, sum(e2e_ms) / len(e2e_ms), e2e_calls, dev)
+    e2e = {"value": e2e_tot / (e2e_ms_max / 1e3), "unit": UNIT,
            "h2d_bytes_per_step": int(trace.sizes.nbytes), "d2h_bytes_per_step": 32,
-           "ms_per_step": float(e2e_t.item())}
+           "ms_per_step": e2e_ms_max}
 
     if rank != 0:
         if dist:
