@@ -16,6 +16,15 @@
 #include "ga_device.cuh"
 #include "ga_internal.h"
 
+// The timed kernel reconverges each warp before every allocator call (a user
+// kernel calling from converged code).  Under independent thread scheduling
+// lanes that leave a divergent call late otherwise enter the next call alone
+// and form their own size-class groups: measured 1.2 lanes per group instead
+// of 2.7 on d4, and 12.6 ms instead of 5.5 ms per step.
+#ifndef GA_TIMED_SYNCWARP
+#define GA_TIMED_SYNCWARP 1
+#endif
+
 namespace {
 
 constexpr uint64_t kNullOff = ~0ull;
@@ -146,8 +155,16 @@ __global__ void __launch_bounds__(256, MINB) k_timed(P al, const uint32_t* __res
     void* held = nullptr;
     for (uint32_t r = 0; r < R; r++) {
         uint32_t n = __ldg(&sizes[(uint64_t)r * T + t]);
+#if GA_TIMED_SYNCWARP
+        // reconverge the warp before each call, as a user kernel calling from
+        // converged code would (T % 32 == 0: every warp runs every round whole)
+        if (T % 32 == 0) __syncwarp();
+#endif
         if (D) {
             if (held) { al.release(held); nfree++; held = nullptr; }
+#if GA_TIMED_SYNCWARP
+            if (T % 32 == 0) __syncwarp();
+#endif
             if (n) { held = al.alloc(n); nm++; nf += held == nullptr; }
         } else if (n) {
             void* p = al.alloc(n);

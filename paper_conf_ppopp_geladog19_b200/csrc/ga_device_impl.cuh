@@ -94,6 +94,9 @@ constexpr int kMaxLevels = 48;
 #ifndef GA_FAST_FA
 #define GA_FAST_FA 1             // 1: that fast path is one fetch-add (no load gate)
 #endif
+#ifndef GA_COUNT_ITERS
+#define GA_COUNT_ITERS 0         // diagnostic: count collective-claim calls / iterations in the repair stats
+#endif
 #ifndef GA_HINT_LDCA
 #define GA_HINT_LDCA 0           // 1: read the per-(arena, class) hint through L1
 #endif
@@ -1256,9 +1259,15 @@ static __device__ __noinline__ uint64_t bin_claim_collective(const ga_desc* h, u
     uint32_t it = 0;                                        // retries move on to the next page
     unsigned unsat = grp;                                   // lanes still without a slot (this lane included)
     GA_DBG_CNT;
+#if GA_COUNT_ITERS
+    if ((int)lane_id() == __ffs(grp) - 1) stat_add(h, kStatRepairNonfull, 1);      // calls (diagnostic build)
+#endif
     for (;;) {
         SPIN_NOTE(dbg_cnt, 10, ((uint64_t)A << 8) | c, unsat);
         const int L = __ffs(unsat) - 1;
+#if GA_COUNT_ITERS
+        if ((int)lane_id() == L) stat_add(h, kStatRepairSummary, 1);               // iterations
+#endif
         uint64_t ch = 0, m = 0;
         if ((int)lane == L) ch = bin_find_chunk(h, A, c, &m);
         ch = __shfl_sync(unsat, ch, L);
