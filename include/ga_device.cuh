@@ -21,6 +21,11 @@
  * with __match_any_sync; one leader per group performs the semaphore and bitmap
  * operations for the whole group (the collective critical sections of
  * P:L1246-1312), so a warp-uniform request costs one semaphore atomic per warp.
+ * Calls are correct from divergent code, but only lanes that arrive together
+ * share a group: under independent thread scheduling, lanes that left an
+ * earlier divergent call late arrive alone.  Reconverge first (__syncwarp())
+ * when the whole warp calls: on the mixed trace that is 2.7 instead of 1.2
+ * lanes per group and 2.3x the throughput.
  *
  * `h` comes from ga_heap_device() (include/ga.h) and is passed by value to the
  * kernel.  Compile with -gencode arch=compute_100a,code=sm_100a.
