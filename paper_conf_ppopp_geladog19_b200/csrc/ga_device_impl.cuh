@@ -94,6 +94,9 @@ constexpr int kMaxLevels = 48;
 #ifndef GA_FAST_FA
 #define GA_FAST_FA 1             // 1: that fast path is one fetch-add (no load gate)
 #endif
+#ifndef GA_CLAIM_ACC
+#define GA_CLAIM_ACC 0           // 1: a page claim keeps claiming in its word until the group is served
+#endif
 #ifndef GA_COUNT_ITERS
 #define GA_COUNT_ITERS 0         // diagnostic: count collective-claim calls / iterations in the repair stats
 #endif
@@ -814,6 +817,31 @@ static __device__ GA_CLAIM_FN uint64_t bin_claim_page(const ga_desc* h, uint64_t
         const uint64_t vm = valid_mask(c, i);
         uint64_t wi_v = i == 0 ? w[0] : i == 1 ? w[1] : i == 2 ? w[2] : w[3];
         uint64_t fr = ~wi_v & vm;
+#if GA_CLAIM_ACC
+        // keep claiming in this word until the whole group is served or the
+        // word is full (a collision costs one more atomicOr, not a new search)
+        uint64_t acc = 0, last = 0;
+        while (fr) {
+            uint64_t m = lowest_bits(fr, need - __popcll(acc));
+            uint64_t old = a_or(&bw[i], m);
+            acc |= m & ~old;
+            last = old | m;
+            if (__popcll(acc) >= need) break;
+            fr = ~last & vm;
+        }
+        if (acc) {
+            if (ld_rlx32(&h->kind[p]) != kind_bin(A, c)) {       // recycled page: undo
+                a_and(&bw[i], ~acc);
+                return 0;
+            }
+            if ((last | ~vm) == ~0ull) {                          // this word is full now
+                ld_bitmap(bw, w);
+                if (page_full(w, c)) nonfull_clear_if_full(h, p, c, A);
+            }
+            *wi = i;
+            return acc;
+        }
+#else
         while (fr) {
             uint64_t m = lowest_bits(fr, need);
             uint64_t old = a_or(&bw[i], m);
@@ -832,6 +860,7 @@ static __device__ GA_CLAIM_FN uint64_t bin_claim_page(const ga_desc* h, uint64_t
             }
             fr = ~(old | m) & vm;
         }
+#endif
     }
     nonfull_clear_if_full(h, p, c, A);
     return 0;
