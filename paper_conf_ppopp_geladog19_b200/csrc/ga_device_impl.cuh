@@ -94,6 +94,9 @@ constexpr int kMaxLevels = 48;
 #ifndef GA_FAST_FA
 #define GA_FAST_FA 1             // 1: that fast path is one fetch-add (no load gate)
 #endif
+#ifndef GA_CLAIM_LOCALMASK
+#define GA_CLAIM_LOCALMASK 0     // 1: a group retries the other non-full pages of its chunk before searching again
+#endif
 #ifndef GA_CLAIM_ACC
 #define GA_CLAIM_ACC 0           // 1: a page claim keeps claiming in its word until the group is served
 #endif
@@ -1287,6 +1290,7 @@ static __device__ __noinline__ uint64_t bin_claim_collective(const ga_desc* h, u
     uint64_t my = kNull;
     uint32_t it = 0;                                        // retries move on to the next page
     unsigned unsat = grp;                                   // lanes still without a slot (this lane included)
+    uint64_t ch = 0, m = 0;                                 // the chunk under claim and its non-full pages
     GA_DBG_CNT;
 #if GA_COUNT_ITERS
     if ((int)lane_id() == __ffs(grp) - 1) stat_add(h, kStatRepairNonfull, 1);      // calls (diagnostic build)
@@ -1297,10 +1301,16 @@ static __device__ __noinline__ uint64_t bin_claim_collective(const ga_desc* h, u
 #if GA_COUNT_ITERS
         if ((int)lane_id() == L) stat_add(h, kStatRepairSummary, 1);               // iterations
 #endif
-        uint64_t ch = 0, m = 0;
-        if ((int)lane == L) ch = bin_find_chunk(h, A, c, &m);
-        ch = __shfl_sync(unsat, ch, L);
-        m = __shfl_sync(unsat, m, L);
+#if GA_CLAIM_LOCALMASK
+        if (m == 0) {                                       // uniform over the group
+#else
+        {
+            ch = 0; m = 0;
+#endif
+            if ((int)lane == L) ch = bin_find_chunk(h, A, c, &m);
+            ch = __shfl_sync(unsat, ch, L);
+            m = __shfl_sync(unsat, m, L);
+        }
         const uint32_t q = __popc(unsat & lanemask_lt());
         const uint32_t np = __popcll(m);
         const uint64_t page = ch * kChunkPages + nth_set(m, (q / per_page + rot + it++) % np);
@@ -1313,6 +1323,14 @@ static __device__ __noinline__ uint64_t bin_claim_collective(const ga_desc* h, u
         wi = __shfl_sync(pg, wi, pl);
         const uint32_t pr = __popc(pg & lanemask_lt());
         if (pr < (uint32_t)__popcll(got)) my = (page << kPageShift) + (uint64_t)(wi * 64 + nth_set(got, pr)) * csz;
+#if GA_CLAIM_LOCALMASK
+        {   // pages that came up short leave the group's local copy of the chunk's
+            // non-full mask: retries go to the other pages before a new search
+            const uint64_t drop = my == kNull ? 1ull << (page & (kChunkPages - 1)) : 0ull;
+            m &= ~(((uint64_t)__reduce_or_sync(unsat, (uint32_t)(drop >> 32)) << 32) |
+                   __reduce_or_sync(unsat, (uint32_t)drop));
+        }
+#endif
         unsat = __ballot_sync(unsat, my == kNull);
         if (my != kNull) break;                             // a satisfied lane leaves the group
     }
