@@ -315,7 +315,7 @@ __global__ void k_bsem_init(uint32_t n_sems, uint64_t* sems, uint32_t variant) {
 // budget 65536 / (256 * minB)); GA_TIMED_OCC=2|4|8 selects.  Default 4 (64
 // registers): measured fastest on d4 (8 forces 32 registers and spills).
 inline int occupancy_target() {
-    static int v = [] { const char* e = getenv("GA_TIMED_OCC"); int x = e ? atoi(e) : 4; return (x == 2 || x == 5 || x == 6 || x == 8) ? x : 4; }();
+    static int v = [] { const char* e = getenv("GA_TIMED_OCC"); int x = e ? atoi(e) : 4; return (x >= 1 && x <= 8 && x != 7) ? x : 4; }();
     return v;
 }
 inline uint32_t nblocks(uint32_t T, uint32_t block) { return (T + block - 1) / block; }
@@ -350,7 +350,9 @@ ga_status ga_trace_timed(ga_heap_t h, ga_stream_t stream, const uint32_t* sizes,
     GaPolicy al{ga_dev_heap{h->ddesc, h->dev.base}};
     cudaStream_t s = (cudaStream_t)stream;
     switch (occupancy_target()) {
+        case 1: k_timed<GaPolicy, 1><<<nblocks(T, block), block, 0, s>>>(al, sizes, R, T, D, counts); break;
         case 2: k_timed<GaPolicy, 2><<<nblocks(T, block), block, 0, s>>>(al, sizes, R, T, D, counts); break;
+        case 3: k_timed<GaPolicy, 3><<<nblocks(T, block), block, 0, s>>>(al, sizes, R, T, D, counts); break;
         case 5: k_timed<GaPolicy, 5><<<nblocks(T, block), block, 0, s>>>(al, sizes, R, T, D, counts); break;
         case 6: k_timed<GaPolicy, 6><<<nblocks(T, block), block, 0, s>>>(al, sizes, R, T, D, counts); break;
         case 8: k_timed<GaPolicy, 8><<<nblocks(T, block), block, 0, s>>>(al, sizes, R, T, D, counts); break;
@@ -414,7 +416,8 @@ ga_status ga_kernel_info(int which, uint32_t block, int* regs, int* blocks_per_s
     if (block == 0) block = 256;
     cudaFuncAttributes a;
     int occ = occupancy_target();
-    const void* f = which == 0 ? (occ == 2 ? (const void*)k_timed<GaPolicy, 2> : occ == 5 ? (const void*)k_timed<GaPolicy, 5>
+    const void* f = which == 0 ? (occ == 1 ? (const void*)k_timed<GaPolicy, 1> : occ == 3 ? (const void*)k_timed<GaPolicy, 3>
+                                  : occ == 2 ? (const void*)k_timed<GaPolicy, 2> : occ == 5 ? (const void*)k_timed<GaPolicy, 5>
                                   : occ == 6 ? (const void*)k_timed<GaPolicy, 6> : occ == 8 ? (const void*)k_timed<GaPolicy, 8>
                                                                                           : (const void*)k_timed<GaPolicy, 4>)
                   : which == 1 ? (const void*)k_churn_round<GaPolicy> : (const void*)k_timed<CudaPolicy, 8>;
