@@ -312,7 +312,7 @@ __global__ void k_bsem_init(uint32_t n_sems, uint64_t* sems, uint32_t variant) {
 }
 
 // resident 256-thread blocks per SM the timed kernel is compiled for (register
-// budget 65536 / (256 * minB)); GA_TIMED_OCC=2|4|8 selects.  Default 4 (64
+// budget 65536 / (256 * minB)); GA_TIMED_OCC=1..6 or 8 selects.  Default 4 (64
 // registers): measured fastest on d4 (8 forces 32 registers and spills).
 inline int occupancy_target() {
     static int v = [] { const char* e = getenv("GA_TIMED_OCC"); int x = e ? atoi(e) : 4; return (x >= 1 && x <= 8 && x != 7) ? x : 4; }();
