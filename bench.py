@@ -386,23 +386,32 @@ def main():
     def step():
         ga.ga_trace_timed(heap.h, stream.cuda_stream, d_sizes.data_ptr(), R, T, D, counts.data_ptr(), args.block)
 
+    def timed_steps(n, cold):
+        """n steps, each bracketed by CUDA events on the heap's stream.  cold: the
+        heap is reset (ga_heap_reset, untimed) before every step, SURVEY 8(d)."""
+        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(n)]
+        for i, (s, e) in enumerate(ev):
+            if cold:
+                heap.reset()                                # untimed, outside the events
+            flush.fill_(i & 7)                              # L2 flush (512 MiB write), outside the events
+            s.record(stream)
+            step()
+            e.record(stream)
+        return ev
+
     for _ in range(args.warmup):
+        heap.reset()
         flush.fill_(1)
         step()
     torch.cuda.synchronize()
     counts.zero_()
-    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
     clocks = Clocks(local)
     clocks.mark()
     if dist:
         dist.barrier()
     torch.cuda.synchronize()
     t_wall = time.perf_counter()
-    for s, e in ev:
-        flush.fill_(s.__hash__() & 7)                      # L2 flush, outside the events
-        s.record(stream)
-        step()
-        e.record(stream)
+    ev = timed_steps(args.steps, cold=True)
     torch.cuda.synchronize()
     if dist:
         dist.barrier()
@@ -411,6 +420,11 @@ def main():
     kern_ms = [s.elapsed_time(e) for s, e in ev]
     ms = sum(kern_ms) / len(kern_ms)
     c = counts.cpu().numpy()
+    # the same steps on a warm heap (no reset: bins and chunks of the previous step reused)
+    counts.zero_()
+    ev_w = timed_steps(args.steps, cold=False)
+    torch.cuda.synchronize()
+    warm_ms = sum(s.elapsed_time(e) for s, e in ev_w) / args.steps
     calls_step = int(c[0] + c[2]) // args.steps
     fails_step = int(c[1]) // args.steps
     ms_max, tot = reduce_over_ranks(dist, ms, calls_step, dev)
@@ -422,6 +436,7 @@ def main():
     from paper_conf_ppopp_geladog19_b200.runner import run_timed_host
     e2e_ms = []
     for i in range(args.warmup + args.steps):
+        heap.reset()
         flush.fill_(2)
         s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         s0.record(stream)
@@ -481,7 +496,9 @@ def main():
            "config": config_of(trace, args), "e2e": e2e, "gpu_launches": args.steps,
            "clocks": clk, "roofline": roofline,
            "calls_per_step": calls_step, "failed_mallocs_per_step": fails_step,
-           "kernel_ms": {"min": min(kern_ms), "max": max(kern_ms)}, "wall_s_timed_region": wall}
+           "kernel_ms": {"min": min(kern_ms), "max": max(kern_ms)},
+           "heap": "cold: ga_heap_reset (untimed) before every step",
+           "warm": {"ms_per_step": warm_ms, "value": calls_step / (warm_ms / 1e3)}, "wall_s_timed_region": wall}
 
     if not args.no_extras:
         # ---- fragmentation (correctness mode: one kernel per round, reserved at boundaries)

@@ -76,7 +76,9 @@ typedef struct ga_desc {
     uint64_t lvl_off[48];     /* word offset of level n in avail                        */
     uint32_t lvl_words[48];   /* u64 words of level n's availability bits               */
     uint32_t* lvl_hint;       /* [48] last level-n word a claim succeeded in            */
-    uint64_t* dbg;            /* GA_DEBUG builds: host-mapped stuck-spin records (or 0) */
+    uint64_t* dbg;            /* host-mapped diagnostic records (ga_debug_attach), or 0  */
+    uint64_t* actr;           /* [n_arenas][8] per-arena call counters: [0] mallocs, [1] frees
+                                 (warp-aggregated; summed by ga_stats)                  */
 } ga_desc;
 
 /* Plain-old-data handle passed BY VALUE to kernels that call ga_malloc /
@@ -86,20 +88,29 @@ typedef struct {
     char* base;               /* pool base (== desc->base)                             */
 } ga_dev_heap;
 
+/* Device counters (failures are the paper's fragmentation
+ * proxy).  Counted on the device by the allocator itself:
+ * n_malloc / n_free per warp call into per-arena words, reserved pages on every
+ * TBuddy allocation / free, the peak with an atomicMax on the growth side. */
 typedef struct {
     uint64_t heap_bytes;          /* usable pool bytes                                     */
     uint64_t metadata_bytes;      /* separate metadata allocation (R-29)                   */
-    uint64_t reserved_bytes;      /* pages held outside the free tree x PAGE (at the call) */
-    uint64_t peak_reserved_bytes; /* max reserved since create/reset (grow paths)          */
+    uint64_t reserved_bytes;      /* pages held outside the free tree x PAGE (device counter) */
+    uint64_t peak_reserved_bytes; /* max of reserved_bytes since create/reset (device atomicMax
+                                     on every allocation from the tree)                    */
+    uint64_t n_malloc;            /* ga_malloc calls, NULL returns and n == 0 included (R-15, R-17) */
+    uint64_t n_free;              /* ga_free calls with p != NULL                          */
     uint64_t n_bin_grow;          /* new bins made (class GROW)                            */
     uint64_t n_chunk_grow;        /* chunks taken from TBuddy                               */
     uint64_t n_bin_reclaim;       /* empty bins returned to their chunk                    */
     uint64_t n_chunk_reclaim;     /* empty chunks returned to TBuddy                       */
     uint64_t n_fallback;          /* group waits degraded to per-lane (R-27)               */
-    uint64_t n_fail;              /* mallocs that returned NULL after every fallback       */
+    uint64_t n_fail;              /* mallocs that returned NULL after every fallback (n > 0) */
     uint64_t n_pending_reclaim;   /* candidate bins not yet reclaimed                      */
     uint64_t n_repair_nonfull;    /* safety net: non-full bits re-published (expected 0)   */
     uint64_t n_repair_summary;    /* safety net: chunk summary bits re-published (expected 0) */
+    uint64_t n_waiter_reclaim;    /* of n_bin_reclaim: bins reclaimed by threads blocked in an
+                                     arena semaphore wait (the delegation of P:L1206-1244)  */
     uint32_t n_arenas;
     uint32_t pad;
 } ga_stats_t;
@@ -116,7 +127,7 @@ ga_status ga_heap_create(int device, ga_stream_t stream, void* buf, size_t bytes
 ga_status ga_heap_destroy(ga_heap_t h);
 /* Return the heap to empty (asynchronous on `stream`); invalidates every pointer. */
 ga_status ga_heap_reset(ga_heap_t h, ga_stream_t stream);
-/* Counters (stream-synchronous D2H copy). */
+/* Counters (stream-ordered D2H copies on `stream`, then a sync of `stream`). */
 ga_status ga_stats(ga_heap_t h, ga_stream_t stream, ga_stats_t* out);
 /* The POD view to pass to kernels. */
 ga_status ga_heap_device(ga_heap_t h, ga_dev_heap* out);
@@ -141,7 +152,7 @@ const char* ga_status_str(ga_status s);
  * Canonical snapshot (logical, little endian; the oracle writes the same format
  * independently, oracle/ga_oracle.c ora_snapshot):
  *   u64 magic "GASNAP01"; u64 heap_bytes; u64 pages; u64 page | (L+1) << 32;
- *   u64 min_class | n_classes << 32 | n_span_classes << 40 | chunk_pages << 48;
+ *   u64 min_class | n_classes << 32 | 5 << 40 (class entries above the bins) | chunk_pages << 48;
  *   u8 kind[pages]: 0x00 free page inside an Available tree node (not its head),
  *                   0x40|n head of an Available node of order n, 0x80|n head of an
  *                   allocated user block of order n, 0x01 tail page of such a block,
@@ -152,9 +163,11 @@ const char* ga_status_str(ga_status s);
  *                   class c: page / (min_class << c); a span of class s:
  *                   chunk_pages >> s), LSB first, padded to bytes;
  *   for each level n = 0..L: 2^(L-n) availability bits, LSB first, padded to bytes;
- *   for each bin class, then each span class: i64 sum over arenas of C, i64 max
- *                   over arenas of |E-R| (the oracle routes span sizes to TBuddy,
- *                   as the paper does, and writes zeros for the span classes);
+ *   for each size class 16 B .. 64 KiB (the 8 bin classes, then 5 entries for
+ *                   4 .. 64 KiB whatever the build routes to spans): i64 sum over
+ *                   arenas of C, i64 max over arenas of |E-R| (zeros for sizes the
+ *                   build -- or the oracle, which routes them to TBuddy as the
+ *                   paper does -- does not serve from spans);
  *   i64 sum of page-semaphore C, i64 max |E-R|;
  *   for each order n = 0..L: i64 C, i64 E-R;
  *   u64 pending reclamation candidates.

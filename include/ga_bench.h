@@ -54,6 +54,15 @@ ga_status ga_trace_timed_host(ga_heap_t h, ga_stream_t stream, const uint32_t* h
                               uint32_t R, uint32_t T, uint32_t D, uint64_t* host_counts,
                               uint32_t block);
 
+/* Device-API edge cases (readings R-15, R-16): thread t < T calls
+ * ga_malloc(sizes[t]) with any u64 size (0 and sizes above the heap return
+ * NULL and are not failures), writes the offset from the heap base to offs[t]
+ * (~0 = NULL), calls ga_free(NULL) (a no-op), and with flags & 1 frees its
+ * block.  sizes, offs: DEVICE u64[T].  T need not be a multiple of 32, so the
+ * last warp runs partial. */
+ga_status ga_edge_calls(ga_heap_t h, ga_stream_t stream, const uint64_t* sizes, uint32_t T,
+                        uint64_t* offs, uint32_t flags, uint32_t block);
+
 /* The same workloads on CUDA's built-in device malloc/free (the baseline of
  * P:L1490-1494).  Set the CUDA heap limit before the first such launch. */
 ga_status ga_cuda_set_heap_limit(size_t bytes);
@@ -96,11 +105,13 @@ typedef struct {
 } ga_bsem_cfg;
 ga_status ga_bsem_bench(ga_stream_t stream, const ga_bsem_cfg* cfg, uint64_t* sems, uint64_t* out);
 
-/* Debug builds (-DGA_DEBUG=1) only: allocate a host-mapped buffer where spin
- * loops that run ~2^18 iterations leave (site, sm|warp|lane, a, b) records,
- * readable while a kernel hangs; *host_records = u64[8 + 4*256], [0] = count.
- * Other builds return GA_EINVAL. */
-ga_status ga_debug_attach(uint64_t** host_records);
+/* Diagnostics: allocate a host-mapped buffer u64[8 + 4*256] (*host_records)
+ * readable while a kernel runs or hangs, and attach it to heap h.  The
+ * allocator's safety net (nfc_repair) leaves one dump of the arena it repaired
+ * in words 1..7 (every build); -DGA_DEBUG=1 builds also record spin loops that
+ * ran ~2^18 iterations as (site, sm|warp|lane, a, b) at [8 + 4i], [0] = count.
+ * The buffer lives until process exit.  GA_EINVAL on null arguments. */
+ga_status ga_debug_attach(ga_heap_t h, uint64_t** host_records);
 
 #ifdef __cplusplus
 }

@@ -40,15 +40,16 @@ def build(force: bool = False) -> str:
 class Layout(ctypes.Structure):
     _fields_ = [("page", ctypes.c_uint32), ("chunk_pages", ctypes.c_uint32),
                 ("min_class", ctypes.c_uint32), ("bin_max", ctypes.c_uint32),
-                ("paper_layout", ctypes.c_uint32), ("snap_span_classes", ctypes.c_uint32)]
+                ("paper_layout", ctypes.c_uint32), ("snap_max_class", ctypes.c_uint32)]
 
 
 # Build layout: 4 KiB pages (R-9), 64-page chunks (R-10),
 # classes 16 B (R-13) .. 2 KiB in bins, >= 4 KiB on the tree (R-12).
-# snap_span_classes is snapshot FORMAT only: the build's span classes (4..64 KiB)
-# have counters in the canonical snapshot; the oracle routes those sizes to
-# TBuddy as the paper does and writes zeros for them.
-BUILD = dict(page=4096, chunk_pages=64, min_class=16, bin_max=2048, paper_layout=0, snap_span_classes=5)
+# snap_max_class is snapshot FORMAT only (include/ga.h): the canonical snapshot
+# has one class counter pair per power of two from 16 B to 64 KiB, the top of
+# BASELINE.json's mixed range (configs[3]); the oracle routes sizes above 2 KiB
+# to TBuddy, as the paper does, and writes zeros for those entries.
+BUILD = dict(page=4096, chunk_pages=64, min_class=16, bin_max=2048, paper_layout=0, snap_max_class=65536)
 # The paper's own layout: 8 B minimum, <= 1 KB in bins with an
 # in-band 128 B header, 2 header bins + 62 tails per chunk, 2 KB -> a 4 KB page.
 PAPER = dict(page=4096, chunk_pages=64, min_class=8, bin_max=1024, paper_layout=1)

@@ -122,10 +122,13 @@ typedef struct {
     uint32_t bin_max;       /* largest bin class (build 2048 B; paper 1024 B, R-12)*/
     uint32_t paper_layout;  /* 1: in-band 128 B bin headers + 2 header bins per
                                chunk + 62 tails (R-11); 0: build     */
-    uint32_t snap_span_classes; /* snapshot FORMAT only: span-class counter pairs
-                               the build's snapshot carries (include/ga.h).  The
-                               oracle serves those sizes from TBuddy, as the paper
-                               does, and writes zeros for them.     */
+    uint32_t snap_max_class;/* snapshot FORMAT only (include/ga.h): the class
+                               section has one counter pair per power of two from
+                               min_class up to this size (65536 = the top of the
+                               16 B - 64 KB mixed range, BASELINE.json configs[3]),
+                               0 = bin classes only.  The oracle serves sizes above
+                               bin_max from TBuddy, as the paper does
+                               (P:L1655-1674), and writes zeros for those entries. */
 } ora_layout;
 
 enum { ST_BUSY = 0, ST_AVAIL = 1, ST_PARTIAL = 2 };   /* node states */
@@ -602,7 +605,9 @@ uint64_t ora_snapshot(const ora_heap* h, uint8_t* out, uint64_t cap) {
     wput_u64(&w, h->heap_bytes);
     wput_u64(&w, h->pages);
     wput_u64(&w, (uint64_t)h->lay.page | ((uint64_t)(h->L + 1) << 32));
-    wput_u64(&w, (uint64_t)h->lay.min_class | ((uint64_t)h->ncls << 32) | ((uint64_t)h->lay.snap_span_classes << 40) |
+    uint32_t extra = h->lay.snap_max_class > h->lay.bin_max
+                     ? (uint32_t)(ilog2_u64(h->lay.snap_max_class) - ilog2_u64(h->lay.bin_max)) : 0;
+    wput_u64(&w, (uint64_t)h->lay.min_class | ((uint64_t)h->ncls << 32) | ((uint64_t)extra << 40) |
                  ((uint64_t)h->lay.chunk_pages << 48));
     /* per-page kind byte */
     uint8_t* kb = (uint8_t*)malloc(h->pages);
@@ -645,7 +650,7 @@ uint64_t ora_snapshot(const ora_heap* h, uint8_t* out, uint64_t cap) {
         int64_t d = h->csem[c].E - h->csem[c].R;
         wput_i64(&w, d < 0 ? -d : d);
     }
-    for (uint32_t s = 0; s < h->lay.snap_span_classes; s++) { wput_i64(&w, 0); wput_i64(&w, 0); }
+    for (uint32_t s = 0; s < extra; s++) { wput_i64(&w, 0); wput_i64(&w, 0); }
     wput_i64(&w, h->psem.C);
     { int64_t d = h->psem.E - h->psem.R; wput_i64(&w, d < 0 ? -d : d); }
     for (int n = 0; n <= h->L; n++) { wput_i64(&w, h->tsem[n].C); wput_i64(&w, h->tsem[n].E - h->tsem[n].R); }

@@ -19,7 +19,7 @@ __all__ = ["lib", "GaError", "Layout", "Stats", "DevHeap", "ga_heap_create", "ga
            "ga_trace_phase", "ga_trace_timed", "ga_trace_timed_host", "ga_cuda_set_heap_limit",
            "ga_cuda_trace_phase", "ga_cuda_trace_timed", "ga_kernel_info", "ga_l2_atomic_bench",
            "ga_bsem_bench", "BsemCfg", "EXPORTED", "GA_TRACE_LOG", "GA_TRACE_TAG",
-           "ga_rcu_workspace_bytes", "ga_rcu_list_removal"]
+           "ga_rcu_workspace_bytes", "ga_rcu_list_removal", "ga_edge_calls"]
 
 GA_TRACE_LOG = 1
 GA_TRACE_TAG = 2
@@ -29,7 +29,7 @@ EXPORTED = ["ga_heap_create", "ga_heap_destroy", "ga_heap_reset", "ga_stats", "g
             "ga_heap_info", "ga_layout", "ga_heap_quiesce", "ga_heap_snapshot", "ga_reserved_pages",
             "ga_status_str", "ga_trace_phase", "ga_trace_timed", "ga_trace_timed_host",
             "ga_cuda_set_heap_limit", "ga_cuda_trace_phase", "ga_cuda_trace_timed",
-            "ga_kernel_info", "ga_l2_atomic_bench", "ga_bsem_bench", "ga_debug_attach",
+            "ga_kernel_info", "ga_l2_atomic_bench", "ga_bsem_bench", "ga_debug_attach", "ga_edge_calls",
             "ga_rcu_workspace_bytes", "ga_rcu_list_removal"]
 
 
@@ -45,9 +45,10 @@ class Layout(ctypes.Structure):
 
 class Stats(ctypes.Structure):
     _fields_ = [(n, ctypes.c_uint64) for n in (
-        "heap_bytes", "metadata_bytes", "reserved_bytes", "peak_reserved_bytes", "n_bin_grow",
+        "heap_bytes", "metadata_bytes", "reserved_bytes", "peak_reserved_bytes", "n_malloc", "n_free", "n_bin_grow",
         "n_chunk_grow", "n_bin_reclaim", "n_chunk_reclaim", "n_fallback", "n_fail",
-        "n_pending_reclaim", "n_repair_nonfull", "n_repair_summary")] + [("n_arenas", ctypes.c_uint32), ("pad", ctypes.c_uint32)]
+        "n_pending_reclaim", "n_repair_nonfull", "n_repair_summary", "n_waiter_reclaim")] + [
+        ("n_arenas", ctypes.c_uint32), ("pad", ctypes.c_uint32)]
 
 
 class DevHeap(ctypes.Structure):
@@ -97,7 +98,8 @@ def lib():
         "ga_kernel_info": [i32, u32, P(i32), P(i32), P(i32)],
         "ga_l2_atomic_bench": [vp, i32, vp, u64, u32, u32, u32, vp],
         "ga_bsem_bench": [vp, P(BsemCfg), vp, vp],
-        "ga_debug_attach": [P(P(u64))],
+        "ga_debug_attach": [vp, P(P(u64))],
+        "ga_edge_calls": [vp, vp, vp, u32, vp, u32, u32],
         "ga_rcu_workspace_bytes": [u32, P(sz)],
         "ga_rcu_list_removal": [vp, u32, u32, vp, vp, sz, u32, u32, vp],
     }
@@ -229,3 +231,7 @@ def ga_rcu_list_removal(stream, n_threads, n_nodes, tags, ws, ws_bytes, delegate
 
 def ga_bsem_bench(stream, cfg: BsemCfg, sems, out):
     _ok(lib().ga_bsem_bench(stream or None, ctypes.byref(cfg), sems, out), "ga_bsem_bench")
+
+
+def ga_edge_calls(h, stream, sizes, T, offs, flags=0, block=256):
+    _ok(lib().ga_edge_calls(h, stream or None, sizes, T, offs, flags, block), "ga_edge_calls")

@@ -22,12 +22,33 @@ NVCC_FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo", "-O3", 
               "-Xcompiler", "-fPIC", "-shared", "-Xptxas", "-warn-spills"]
 
 
-def _stale() -> bool:
-    if not os.path.exists(LIB):
+def _stale(lib: str = LIB) -> bool:
+    if not os.path.exists(lib):
         return True
-    t = os.path.getmtime(LIB)
+    t = os.path.getmtime(lib)
     srcs = [os.path.join(CSRC, f) for f in DEPS] + [os.path.join(INCLUDE, f) for f in HEADERS]
     return any(os.path.getmtime(s) > t for s in srcs)
+
+
+# Build variants the tests load through GA_LIB (each a complete libga.so):
+#   nspan0 -- GA_NSPAN=0, the paper's routing (every size above the bins on
+#             TBuddy), run by the parity suite (tests/test_gpu_variants.py).
+VARIANTS = {"nspan0": ("GA_NSPAN=0",)}
+
+
+def variant_path(name: str) -> str:
+    return os.path.join(PKG, f"libga_{name}.so")
+
+
+def build_variants(force: bool = False) -> dict:
+    """Compile every VARIANTS entry next to libga.so (if missing or stale)."""
+    out = {}
+    for name, defines in VARIANTS.items():
+        path = variant_path(name)
+        if force or not os.path.exists(path) or _stale(path):
+            build(defines=defines, out=path)
+        out[name] = path
+    return out
 
 
 def build(force: bool = False, verbose: bool = False, defines=(), out: str | None = None) -> str:
@@ -54,3 +75,5 @@ def build(force: bool = False, verbose: bool = False, defines=(), out: str | Non
 if __name__ == "__main__":
     build(force=True, verbose="-v" in sys.argv)
     print(LIB)
+    for path in build_variants(force=True).values():
+        print(path)

@@ -176,6 +176,17 @@ __global__ void __launch_bounds__(256, MINB) k_timed(P al, const uint32_t* __res
     flush_counts(counts, nm, nf, nfree, 0);
 }
 
+// device-API edge cases (R-15, R-16): any u64 size, free(NULL), partial warps
+__global__ void __launch_bounds__(256) k_edge(GaPolicy al, const uint64_t* sizes, uint32_t T, uint64_t* offs,
+                                              uint32_t flags) {
+    uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= T) return;
+    void* p = al.alloc(sizes[t]);
+    offs[t] = al.off(p);
+    al.release(nullptr);                                      // R-16: a no-op
+    if ((flags & 1) && p) al.release(p);
+}
+
 // --------------------------------------------------------------------------
 // L2-atomic peak microbenchmark
 // --------------------------------------------------------------------------
@@ -330,6 +341,7 @@ ga_status ga_trace_phase(ga_heap_t h, ga_stream_t stream, const uint32_t* sizes,
                          uint32_t flags, uint32_t block) {
     if (!h || !sizes || !held || !counts || T == 0 || D > 1) return GA_EINVAL;
     if (block == 0) block = 256;
+    DeviceGuard g(h->device);
     GaPolicy al{ga_dev_heap{h->ddesc, h->dev.base}};
     cudaStream_t s = (cudaStream_t)stream;
     if (!(flags & GA_TRACE_LOG)) log = nullptr;
@@ -347,6 +359,7 @@ ga_status ga_trace_timed(ga_heap_t h, ga_stream_t stream, const uint32_t* sizes,
                          uint64_t* counts, uint32_t block) {
     if (!h || !sizes || !counts || T == 0 || D > 1) return GA_EINVAL;
     if (block == 0) block = 256;
+    DeviceGuard g(h->device);
     GaPolicy al{ga_dev_heap{h->ddesc, h->dev.base}};
     cudaStream_t s = (cudaStream_t)stream;
     switch (occupancy_target()) {
@@ -364,6 +377,7 @@ ga_status ga_trace_timed(ga_heap_t h, ga_stream_t stream, const uint32_t* sizes,
 ga_status ga_trace_timed_host(ga_heap_t h, ga_stream_t stream, const uint32_t* host_sizes, uint32_t R, uint32_t T,
                               uint32_t D, uint64_t* host_counts, uint32_t block) {
     if (!h || !host_sizes || !host_counts || T == 0 || D > 1) return GA_EINVAL;
+    DeviceGuard g(h->device);
     cudaStream_t s = (cudaStream_t)stream;
     size_t sz = (size_t)R * T * 4;
     size_t need = sz + 256 + 64;
@@ -381,6 +395,16 @@ ga_status ga_trace_timed_host(ga_heap_t h, ga_stream_t stream, const uint32_t* h
     if (st != GA_OK) return st;
     if (cudaMemcpyAsync(host_counts, d_counts, 32, cudaMemcpyDeviceToHost, s) != cudaSuccess) return GA_ECUDA;
     return cudaStreamSynchronize(s) == cudaSuccess ? GA_OK : GA_ECUDA;
+}
+
+ga_status ga_edge_calls(ga_heap_t h, ga_stream_t stream, const uint64_t* sizes, uint32_t T, uint64_t* offs,
+                        uint32_t flags, uint32_t block) {
+    if (!h || !sizes || !offs || T == 0) return GA_EINVAL;
+    if (block == 0) block = 256;
+    DeviceGuard g(h->device);
+    k_edge<<<nblocks(T, block), block, 0, (cudaStream_t)stream>>>(GaPolicy{ga_dev_heap{h->ddesc, h->dev.base}},
+                                                                  sizes, T, offs, flags);
+    return launched();
 }
 
 ga_status ga_cuda_set_heap_limit(size_t bytes) {
@@ -437,13 +461,18 @@ ga_status ga_l2_atomic_bench(ga_stream_t stream, int pattern, uint64_t* d_buf, u
     return launched();
 }
 
-ga_status ga_debug_attach(uint64_t** host_records) {
-    if (!host_records) return GA_EINVAL;
+ga_status ga_debug_attach(ga_heap_t h, uint64_t** host_records) {
+    if (!h || !host_records) return GA_EINVAL;
+    DeviceGuard g(h->device);
     void* hp = nullptr;
     if (cudaHostAlloc(&hp, 8 * (8 + 4 * 256), cudaHostAllocMapped) != cudaSuccess) return GA_ENOMEM;
     memset(hp, 0, 8 * (8 + 4 * 256));
     void* dp = nullptr;
     if (cudaHostGetDevicePointer(&dp, hp, 0) != cudaSuccess) return GA_ECUDA;
+    // the heap descriptor (every translation unit's allocator code reads it) ...
+    h->dev.dbg = (uint64_t*)dp;
+    if (cudaMemcpy(&h->ddesc->dbg, &h->dev.dbg, sizeof(uint64_t*), cudaMemcpyHostToDevice) != cudaSuccess) return GA_ECUDA;
+    // ... and GA_DEBUG builds' spin-loop records (this translation unit)
     if (cudaMemcpyToSymbol(ga::g_ga_dbg, &dp, sizeof dp) != cudaSuccess) return GA_ECUDA;
     *host_records = (uint64_t*)hp;
     return GA_OK;

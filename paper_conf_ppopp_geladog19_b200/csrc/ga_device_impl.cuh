@@ -79,26 +79,11 @@ constexpr int kMaxLevels = 48;
 #ifndef GA_TREE_SPIN_CAP
 #define GA_TREE_SPIN_CAP 256     // max __nanosleep backoff (ns) of a blocked TBuddy wait
 #endif
-#ifndef GA_OPT_LOAD_GATED
-#define GA_OPT_LOAD_GATED 0      // 1: optimistic (TBuddy) waits decide on a plain load first
-#endif
-#ifndef GA_MERGE_PRELOAD
-#define GA_MERGE_PRELOAD 1       // 1: try-wait loads the word before its fetch-add
-#endif
 #ifndef GA_INL_CLAIM
 #define GA_INL_CLAIM 1           // 1: inline the hint lookup and page claim into the collective claim
 #endif
-#ifndef GA_INL_WAIT
-#define GA_INL_WAIT 1            // 1: the arena-semaphore fast path inline at the malloc entry
-#endif
-#ifndef GA_FAST_FA
-#define GA_FAST_FA 1             // 1: that fast path is one fetch-add (no load gate)
-#endif
 #ifndef GA_CLAIM_LOCALMASK
 #define GA_CLAIM_LOCALMASK 0     // 1: a group retries the other non-full pages of its chunk before searching again
-#endif
-#ifndef GA_CLAIM_ACC
-#define GA_CLAIM_ACC 0           // 1: a page claim keeps claiming in its word until the group is served
 #endif
 #ifndef GA_COUNT_ITERS
 #define GA_COUNT_ITERS 0         // diagnostic: count collective-claim calls / iterations in the repair stats
@@ -115,10 +100,38 @@ constexpr uint32_t kReclaimKeep = 64;           // free slots a delegated reclai
 
 enum { kStatBinGrow = 0, kStatChunkGrow, kStatBinReclaim, kStatChunkReclaim, kStatFallback,
        kStatFail, kStatRepairNonfull, kStatRepairSummary, kNumStats };
+// device words of the reserved-page counter and its peak (own 32 B sectors of
+// the stats block), and the per-arena call counters (ga_stats_t)
+constexpr int kStatReserved = 8, kStatPeakReserved = 12, kStatWords = 16;
+constexpr int kStatWaiterReclaim = 9;           // bins reclaimed by threads blocked in a wait
+constexpr int kActrStride = 8;                  // u64 words per arena: [0] mallocs, [1] frees
 
 static __device__ __forceinline__ uint32_t lane_id() { uint32_t r; asm volatile("mov.u32 %0, %%laneid;" : "=r"(r)); return r; }
 static __device__ __forceinline__ uint32_t lanemask_lt() { uint32_t r; asm volatile("mov.u32 %0, %%lanemask_lt;" : "=r"(r)); return r; }
 static __device__ __forceinline__ uint32_t smid() { uint32_t r; asm volatile("mov.u32 %0, %%smid;" : "=r"(r)); return r; }
+// Warp masks for the *_sync intrinsics, made opaque to the compiler's
+// uniformity analysis.  Lanes that call the allocator from divergent code
+// compute their masks in separate groups (each from its own __activemask()),
+// and the groups can be merged at a later convergence barrier (BSYNC).  A mask
+// the compiler believes warp-uniform (a ballot result) is then read through a
+// uniform register (R2UR) as if every co-active lane held the same value: on
+// sm_100a some merged lanes skipped a __syncwarp as "already converged" while
+// the others waited in its divergent path -- a hang at two different WARPSYNCs
+// (cuda-gdb, tests/test_gpu_edge.py).  Opaque masks make the compiler check
+// uniformity (REDUX.OR + R2UR P) before shfl / vote / match and take the
+// per-lane collective path (WARPSYNC.COLLECTIVE) when they differ.
+// __syncwarp(mask) is lowered through R2UR whatever the mask, so the allocator
+// does not use it: a following match / ballot on the same mask is the
+// execution barrier, and warp_release() is the publication barrier.
+static __device__ __forceinline__ unsigned opaque_mask(unsigned m) { asm volatile("" : "+r"(m)); return m; }
+static __device__ __forceinline__ unsigned active_lanes() { return opaque_mask(__activemask()); }
+// Every lane of `grp` has performed its prior writes at gpu scope (fence) and
+// reached this point (ballot) before any lane of grp continues: a leader's
+// release signal that follows publishes every lane's writes.
+static __device__ __forceinline__ void warp_release(unsigned grp) {
+    asm volatile("fence.acq_rel.gpu;" ::: "memory");
+    (void)__ballot_sync(grp, 1);
+}
 
 static __device__ __forceinline__ uint64_t ld_rlx(const uint64_t* p) {
     uint64_t v; asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory"); return v;
@@ -162,14 +175,26 @@ static __device__ __forceinline__ uint64_t recheck_read(uint64_t* p) {
 #endif
 }
 static __device__ __forceinline__ void stat_add(const ga_desc* h, int i, uint64_t v) { a_add(&h->stats[i], v); }
+// pages leaving (d > 0) or returning to (d < 0) the free tree; the peak is an
+// atomicMax on the growth side only (SURVEY 8(a) a10, 8(d) "peak_reserved_X")
+static __device__ __noinline__ void reserve_add(const ga_desc* h, int64_t d) {
+    if (d <= 0) {
+        asm volatile("red.relaxed.gpu.global.add.u64 [%0], %1;" :: "l"(&h->stats[kStatReserved]), "l"((uint64_t)d) : "memory");
+        return;
+    }
+    const uint64_t v = a_add(&h->stats[kStatReserved], (uint64_t)d) + (uint64_t)d;
+    if (v > ld_rlx(&h->stats[kStatPeakReserved])) atomicMax((unsigned long long*)&h->stats[kStatPeakReserved], (unsigned long long)v);
+}
 
 // GA_DEBUG builds: a spin loop that runs ~2^20 times records (site, ids, a, b)
 // into host-mapped memory, readable while a kernel hangs (tools/hang_probe.py)
 #ifndef GA_DEBUG
 #define GA_DEBUG 0
 #endif
-// host-mapped diagnostics (ga_debug_attach); null unless attached.  Release
-// builds only touch it on the cold safety-net path (nfc_repair).
+// host-mapped records of GA_DEBUG builds' spin loops (ga_debug_attach sets
+// ga_bench.cu's copy; those loops have no heap descriptor at hand).  The
+// safety-net dump in nfc_repair reads the descriptor's dbg field instead, so it
+// works from every translation unit.
 static __device__ uint64_t* g_ga_dbg;
 #if GA_DEBUG
 #define SPIN_NOTE(cnt, site, a, b) spin_note((cnt), (site), (uint64_t)(a), (uint64_t)(b))
@@ -258,137 +283,123 @@ static __device__ __forceinline__ void bsem_signal_after_rmw(uint64_t* s, uint32
     asm volatile("red.relaxed.gpu.global.add.u64 [%0], %1;" :: "l"(s), "l"((uint64_t)N << 32) : "memory");
 }
 
-// try-wait (R-7): C -= N iff C >= N.  One fetch-add: subtract,
-// and give the units back if the pre-image was short.
-// one fetch-add, no pre-load (callers that expect success, e.g. a merge whose
-// buddy bit was just seen set)
-static __device__ __forceinline__ bool bsem_trywait_direct(uint64_t* s, uint32_t N) {
-    const uint64_t dn = (uint64_t)N << 32;
-    uint64_t old = a_add(s, (uint64_t)0 - dn);
-    if (sem_C(old) >= (int32_t)N) return true;
-    a_add(s, dn);
+// Conservative in-flight encoding (R-35; model-checked by
+// oracle/bsem.py explore_gpu, tests/test_oracle_bsem.py).  A fetch-add that
+// speculates moves units from C into D instead of removing them: (C -= N,
+// D += N) keeps C + D.  While it is in flight the word therefore only shows
+// LESS value (C) and MORE cover (C + D) than the state with every decided
+// operation applied, so no other thread can take units that are not there or
+// decide GROW when that state would not.  Each speculation is settled by one
+// more add: a repayment of D, or the reverse move.
+static __device__ __forceinline__ uint64_t dCD(int32_t dc, int32_t dd) {
+    return ((uint64_t)(int64_t)dc << 32) + (uint64_t)(int64_t)dd;
+}
+static __device__ __forceinline__ void red_rlx(uint64_t* s, uint64_t v) {
+    asm volatile("red.relaxed.gpu.global.add.u64 [%0], %1;" :: "l"(s), "l"(v) : "memory");
+}
+
+// try-wait (R-7): C -= N iff C >= N (+ keep units stay behind).
+// direct: no pre-load (callers that expect success, e.g. a merge whose buddy
+// bit was just seen set).
+static __device__ __forceinline__ bool bsem_trywait_direct(uint64_t* s, uint32_t N, uint32_t keep = 0) {
+    uint64_t old = a_add(s, dCD(-(int32_t)N, (int32_t)N));
+    if (sem_C(old) >= (int32_t)(N + keep)) { red_rlx(s, dCD(0, -(int32_t)N)); return true; }
+    red_rlx(s, dCD((int32_t)N, -(int32_t)N));
     return false;
 }
 static __device__ __forceinline__ bool bsem_trywait(uint64_t* s, uint32_t N, uint32_t keep = 0) {
-    // keep: succeed only if at least `keep` further units stay behind
     if (sem_C(ld_rlx(s)) < (int32_t)(N + keep)) return false;
-    const uint64_t dn = (uint64_t)N << 32;
-    uint64_t old = a_add(s, (uint64_t)0 - dn);
-    if (sem_C(old) >= (int32_t)(N + keep)) return true;
-    a_add(s, dn);
+    return bsem_trywait_direct(s, N, keep);
+}
+
+// Fast acquire: one fetch-add (C -= N, D += N).  ACQUIRED iff the pre-image
+// shows C >= N and C + D >= N (Alg. 1 tests growth first); the speculation is
+// then settled by a repayment red (D -= N).  Otherwise the move is reversed and
+// the returned word (*w) seeds the exact CAS loop.
+static __device__ __forceinline__ bool bsem_fast_acquire(uint64_t* s, uint32_t N, uint64_t* w) {
+    const uint64_t d = dCD(-(int32_t)N, (int32_t)N);
+    const uint64_t old = a_add(s, d);
+    if (sem_C(old) >= (int32_t)N && (int64_t)sem_C(old) + sem_D(old) >= (int64_t)N) {
+        red_rlx(s, dCD(0, -(int32_t)N));
+        return true;
+    }
+    const uint64_t back = dCD((int32_t)N, -(int32_t)N);
+    *w = a_add(s, back) + back;
     return false;
 }
 
-// Alg. 1 core (documentation at bsem_wait below).
-template <bool kExact, class Spin>
-static __device__ __noinline__ int bsem_wait_impl(uint64_t* s, uint32_t N, uint32_t B, Spin spin) {
+// Alg. 1 as a CAS loop on the packed word, starting from the
+// caller's copy w.  One CAS decides among the three branches on the current
+// word; a blocked waiter runs `spin()` -- the delegated work of Sec. 4.2.1 --
+// between polls.  Reading R-2: keep waiting while C < N and C + D >= 0.
+template <class Spin>
+static __device__ __noinline__ int bsem_wait_cas(uint64_t* s, uint32_t N, uint32_t B, Spin spin, uint64_t w) {
     GA_DBG_CNT;
-    const uint64_t dn = (uint64_t)N << 32;
-    uint64_t w;
-    if (kExact) {
-        // Fast path: a plain load says the units are there -> one fetch-add.
-        // If it raced (pre-image short), give them back and run the exact form.
-        w = ld_rlx(s);
-        if (sem_C(w) >= (int32_t)N) {
-            uint64_t old = a_add(s, (uint64_t)0 - dn);
-            if (sem_C(old) >= (int32_t)N) return kAcquired;
-            w = a_add(s, dn) + dn;
-        }
-        // Exact Alg. 1: one CAS decides among the three branches on the current word.
-        for (;;) {
-            int32_t C = sem_C(w), D = sem_D(w);
-            uint64_t nw;
-            int res;
-            if ((int64_t)C + D < (int64_t)N) { nw = w + (uint64_t)(B - N); res = kGrow; }         // E += B - N
-            else if (C >= (int32_t)N) { nw = w - dn; res = kAcquired; }                        // C -= N
-            else { nw = w - (uint64_t)N; res = kBlocked; }                                      // R += N
-            uint64_t old = a_cas(s, w, nw);
-            if (old != w) { w = old; continue; }
-            if (res != kBlocked) return res;
-            uint32_t ns = 64;
-            for (;;) {                                                                          // R-2
-                w = ld_rlx(s);
-                if (!(sem_C(w) < (int32_t)N && (int64_t)sem_C(w) + sem_D(w) >= 0)) break;
-                spin();
-                SPIN_NOTE(dbg_cnt, 1, (uint64_t)(uintptr_t)s, w);
-                __nanosleep(ns);
-                if (ns < 2048) ns <<= 1;
-            }
-            w = a_add(s, (uint64_t)N) + (uint64_t)N;                                            // R -= N
-        }
-    }
-#if GA_OPT_LOAD_GATED
-    // Optimistic form, load-gated: each decision is taken on a plain load and
-    // applied with ONE fetch-add; C is only decremented when the load showed
-    // enough units, so a hot order semaphore is not disturbed by waiters.
-    //   load C >= N          -> fetch-add C -= N (ACQUIRED unless raced: give back)
-    //   load C + D < N       -> fetch-add E += B - N: GROW
-    //   otherwise            -> fetch-add R += N, spin (R-2), R -= N, re-decide
-    // A stale load can only over-produce (an extra split stays inside the tree)
-    // or send a reserved waiter straight back to re-decide; it never over-grants.
-    w = ld_rlx(s);
     for (;;) {
-        if (sem_C(w) >= (int32_t)N) {
-            uint64_t old = a_add(s, (uint64_t)0 - dn);
-            if (sem_C(old) >= (int32_t)N) return kAcquired;
-            w = a_add(s, dn) + dn;
-            continue;
-        }
-        if ((int64_t)sem_C(w) + sem_D(w) < (int64_t)N) {
-            a_add(s, (uint64_t)(B - N));                                                        // E += B - N
-            return kGrow;
-        }
-        w = a_add(s, (uint64_t)0 - (uint64_t)N) - (uint64_t)N;                                  // R += N
-        uint32_t ns = 32;
-        while (sem_C(w) < (int32_t)N && (int64_t)sem_C(w) + sem_D(w) >= 0) {                    // R-2
-            spin();
-            SPIN_NOTE(dbg_cnt, 2, (uint64_t)(uintptr_t)s, w);
-            __nanosleep(ns);
-            if (ns < GA_TREE_SPIN_CAP) ns <<= 1;
+        int32_t C = sem_C(w), D = sem_D(w);
+        uint64_t nw;
+        int res;
+        if ((int64_t)C + D < (int64_t)N) { nw = w + (uint64_t)(B - N); res = kGrow; }          // E += B - N
+        else if (C >= (int32_t)N) { nw = w - ((uint64_t)N << 32); res = kAcquired; }        // C -= N
+        else { nw = w - (uint64_t)N; res = kBlocked; }                                       // R += N
+        uint64_t old = a_cas(s, w, nw);
+        if (old != w) { w = old; continue; }
+        if (res != kBlocked) return res;
+        uint32_t ns = 64;
+        for (;;) {                                                                           // R-2
             w = ld_rlx(s);
+            if (!(sem_C(w) < (int32_t)N && (int64_t)sem_C(w) + sem_D(w) >= 0)) break;
+            spin();
+            SPIN_NOTE(dbg_cnt, 1, (uint64_t)(uintptr_t)s, w);
+            __nanosleep(ns);
+            if (ns < 2048) ns <<= 1;
         }
-        w = a_add(s, (uint64_t)N) + (uint64_t)N;                                                // R -= N
+        w = a_add(s, (uint64_t)N) + (uint64_t)N;                                             // R -= N
     }
-#else
-    // Optimistic form: one fetch-add C -= N decides on the pre-image.
-    //   pre C >= N           -> ACQUIRED (one atomic, no retry)
-    //   pre C + D < N        -> GROW: give C back, E += B - N
-    //   otherwise            -> reserve: give C back, R += N (C + D unchanged), spin
-    // Reservation conversions keep C + D exact; an in-flight GROW conversion hides
-    // its units for one round trip, so others may over-produce (never over-grant).
+}
+
+// Alg. 1 for arena semaphores (class and page: an extra batch costs real
+// pages).  Returns kAcquired (0) or kGrow (-1; the caller must produce B
+// units, keep N and signal(B - N, B - N), or signal(0, B - N) on failure,
+// P:L756-764).  A plain load gates the fast acquire.
+template <class Spin>
+static __device__ __forceinline__ int bsem_wait(uint64_t* s, uint32_t N, uint32_t B, Spin spin) {
+    uint64_t w = ld_rlx(s);
+    if (sem_C(w) >= (int32_t)N && (int64_t)sem_C(w) + sem_D(w) >= (int64_t)N && bsem_fast_acquire(s, N, &w))
+        return kAcquired;
+    return bsem_wait_cas(s, N, B, spin, w);
+}
+
+// Alg. 1 for TBuddy order semaphores, in fetch-adds (no CAS retries on the few
+// hot order words).  The first fetch-add (C -= N, D += B) covers every outcome
+// conservatively; the pre-image decides in Alg. 1's order and one more add
+// settles it:
+//   pre C + D < N   -> GROW:     (C += N, D -= N)       net E += B - N
+//   pre C >= N      -> ACQUIRED: (D -= B)               net C -= N
+//   otherwise       -> reserve:  (C += N, D -= N + B)   net R += N; spin (R-2),
+//                      then R -= N and decide again.
+template <class Spin>
+static __device__ __noinline__ int bsem_wait_fast(uint64_t* s, uint32_t N, uint32_t B, Spin spin) {
+    GA_DBG_CNT;
+    const uint64_t first = dCD(-(int32_t)N, (int32_t)B);
     for (;;) {
-        uint64_t old = a_add(s, (uint64_t)0 - dn);
-        int32_t C = sem_C(old), D = sem_D(old);
-        if (C >= (int32_t)N) return kAcquired;
-        if ((int64_t)C + D < (int64_t)N) {
-            a_add(s, dn + (uint64_t)(B - N));                                                   // C += N, E += B - N
-            return kGrow;
-        }
-        w = a_add(s, dn - (uint64_t)N) + dn - (uint64_t)N;                                     // C += N, R += N
+        const uint64_t old = a_add(s, first);
+        const int32_t C = sem_C(old), D = sem_D(old);
+        if ((int64_t)C + D < (int64_t)N) { red_rlx(s, dCD((int32_t)N, -(int32_t)N)); return kGrow; }
+        if (C >= (int32_t)N) { red_rlx(s, dCD(0, -(int32_t)B)); return kAcquired; }
+        const uint64_t res = dCD((int32_t)N, -(int32_t)(N + B));
+        uint64_t w = a_add(s, res) + res;
         uint32_t ns = 32;
-        while (sem_C(w) < (int32_t)N && (int64_t)sem_C(w) + sem_D(w) >= 0) {                    // R-2
+        while (sem_C(w) < (int32_t)N && (int64_t)sem_C(w) + sem_D(w) >= 0) {                  // R-2
             spin();
             SPIN_NOTE(dbg_cnt, 3, (uint64_t)(uintptr_t)s, w);
             __nanosleep(ns);
             if (ns < GA_TREE_SPIN_CAP) ns <<= 1;
             w = ld_rlx(s);
         }
-        a_add(s, (uint64_t)N);                                                                  // R -= N
+        red_rlx(s, (uint64_t)N);                                                             // R -= N
     }
-#endif
 }
-// Alg. 1.  Returns kAcquired (0) or kGrow (-1; the caller must
-// produce B units, keep N and signal(B - N, B - N), or signal(0, B - N) on
-// failure).  While blocked it runs `spin()` -- the delegated work
-// of Sec. 4.2.1 -- between polls.  Reading R-2: keep waiting while
-// C < N and R <= C + E, i.e. C < N and C + D >= 0.
-// bsem_wait: exact growth decisions (arena class / page semaphores: an extra
-//   batch costs real pages); bsem_wait_fast: optimistic (TBuddy orders: an extra
-//   split stays available inside the tree).  DESIGN.md "Semaphore word".
-template <class Spin>
-static __device__ __forceinline__ int bsem_wait(uint64_t* s, uint32_t N, uint32_t B, Spin spin) { return bsem_wait_impl<true>(s, N, B, spin); }
-template <class Spin>
-static __device__ __forceinline__ int bsem_wait_fast(uint64_t* s, uint32_t N, uint32_t B, Spin spin) { return bsem_wait_impl<false>(s, N, B, spin); }
 struct NoSpin { __device__ void operator()() const {} };
 
 // ---------------------------------------------------------------------------
@@ -546,6 +557,7 @@ static __device__ __noinline__ int64_t tree_alloc_one(const ga_desc* h, int o) {
     uint64_t got = tree_claim_word(h, m, 1, scatter_seed(), &wj);
     uint64_t x = wj * 64 + (uint64_t)(__ffsll((long long)got) - 1);
     for (int k = m - 1; k >= o; k--) { x = 2 * x; tree_publish(h, k, x + 1, 1); }
+    reserve_add(h, (int64_t)1 << o);
     return (int64_t)x;
 }
 
@@ -556,6 +568,7 @@ static __device__ __noinline__ int64_t tree_alloc_one(const ga_desc* h, int o) {
 static __device__ __noinline__ void tree_free(const ga_desc* h, int n, uint64_t x) {
     GA_DBG_CNT;
     uint32_t ns = 32;
+    reserve_add(h, -((int64_t)1 << n));
     for (;;) {
         HB3 b = level_hb(h, n);
         uint64_t* wp = &b.w0[x >> 6];
@@ -563,7 +576,7 @@ static __device__ __noinline__ void tree_free(const ga_desc* h, int n, uint64_t 
         bool root = (n >= (int)h->L) || !node_inside(h, n, x ^ 1);
         uint64_t w = ld_rlx(wp);
         if (!root && (w & yb)) {
-            if (GA_MERGE_PRELOAD ? bsem_trywait(tsem_ptr(h, n), 1) : bsem_trywait_direct(tsem_ptr(h, n), 1)) {
+            if (bsem_trywait(tsem_ptr(h, n), 1)) {
                 uint64_t old = a_and(wp, ~yb);
                 if (old & yb) {                               // merged: free the parent at n + 1
                     if (old == yb) hb3_up_clear(b, (uint32_t)(x >> 6));
@@ -625,11 +638,14 @@ static __device__ __forceinline__ bool page_full(const uint64_t w[4], int c) {
     return true;
 }
 
-static __device__ void reclaim_arena(const ga_desc* h, uint32_t A, int budget, uint32_t keep);
-// delegated work run by threads blocked in an arena semaphore wait (Sec. 4.2.1)
+static __device__ int reclaim_arena(const ga_desc* h, uint32_t A, int budget, uint32_t keep);
+// delegated work run by threads blocked in an arena semaphore wait (Sec. 4.2.1);
+// what they reclaim is counted (ga_stats n_waiter_reclaim)
 struct ArenaSpin {
     const ga_desc* h; uint32_t A;
-    __device__ void operator()() const { reclaim_arena(h, A, 4, kReclaimKeep); }
+    __device__ void operator()() const {
+        if (const int n = reclaim_arena(h, A, 4, kReclaimKeep)) stat_add(h, kStatWaiterReclaim, (uint64_t)n);
+    }
 };
 
 // Data bit `bit` of *data (a per-chunk word: non-full pages, reclaim
@@ -718,8 +734,14 @@ static __device__ __noinline__ uint64_t page_claim(const ga_desc* h, uint32_t A,
                     uint64_t got = m & ~old;
                     u = old | m;
                     if (!got) continue;
-                    if (ld_rlx32(&h->chunk_owner[ch]) != A + 1) {  // recycled chunk: undo
+                    if (const uint32_t o = ld_rlx32(&h->chunk_owner[ch]); o != A + 1) {
+                        // recycled chunk (now o's): undo, then re-publish the chunk
+                        // in its owner's free-page summary -- a claimer of o may
+                        // have seen our bits, found the chunk full and cleared it.
+                        // Our bits kept the chunk from being released meanwhile,
+                        // so o is its owner.
                         a_and(&h->chunk_used[ch], ~got);
+                        if (o != 0) hb3_set(arena_hb(h, o - 1, kAhbFpc), (uint64_t)ch);
                         break;
                     }
                     if (u == ~0ull) hb3_clear_summarised(fb, ch, &h->chunk_used[ch], ~0ull);
@@ -793,6 +815,16 @@ static __device__ __forceinline__ void bin_init(const ga_desc* h, uint64_t p, ui
     if (take < slots_of(c)) nonfull_set(h, p, c, A);
 }
 
+// Give back slots `got` of word i of page p, taken by a stale claimer after p
+// became a bin of another incarnation (kind k2), and re-publish p for it.
+static __device__ __noinline__ void undo_claim(const ga_desc* h, uint64_t p, int i, uint64_t got, uint32_t k2) {
+    a_and(&page_bits(h, p)[i], ~got);
+    if ((k2 & 0xC0000000u) == kKindBin) {
+        nonfull_set(h, p, (int)(k2 & 0xFF), (k2 >> 8) & 0xFFFFu);
+        mark_candidate(h, p, (k2 >> 8) & 0xFFFFu);
+    }
+}
+
 // Claim up to `need` slots of page p (an (A, c) bin) from one bitmap word with
 // one atomicOr.  Returns the claimed mask (word in *wi); 0 if none.  The page
 // kind and the bitmap are loaded together (independent round trips), and the
@@ -820,38 +852,16 @@ static __device__ GA_CLAIM_FN uint64_t bin_claim_page(const ga_desc* h, uint64_t
         const uint64_t vm = valid_mask(c, i);
         uint64_t wi_v = i == 0 ? w[0] : i == 1 ? w[1] : i == 2 ? w[2] : w[3];
         uint64_t fr = ~wi_v & vm;
-#if GA_CLAIM_ACC
-        // keep claiming in this word until the whole group is served or the
-        // word is full (a collision costs one more atomicOr, not a new search)
-        uint64_t acc = 0, last = 0;
-        while (fr) {
-            uint64_t m = lowest_bits(fr, need - __popcll(acc));
-            uint64_t old = a_or(&bw[i], m);
-            acc |= m & ~old;
-            last = old | m;
-            if (__popcll(acc) >= need) break;
-            fr = ~last & vm;
-        }
-        if (acc) {
-            if (ld_rlx32(&h->kind[p]) != kind_bin(A, c)) {       // recycled page: undo
-                a_and(&bw[i], ~acc);
-                return 0;
-            }
-            if ((last | ~vm) == ~0ull) {                          // this word is full now
-                ld_bitmap(bw, w);
-                if (page_full(w, c)) nonfull_clear_if_full(h, p, c, A);
-            }
-            *wi = i;
-            return acc;
-        }
-#else
         while (fr) {
             uint64_t m = lowest_bits(fr, need);
             uint64_t old = a_or(&bw[i], m);
             uint64_t got = m & ~old;
             if (got) {
-                if (ld_rlx32(&h->kind[p]) != kind_bin(A, c)) {   // recycled page: undo
-                    a_and(&bw[i], ~got);
+                if (const uint32_t k2 = ld_rlx32(&h->kind[p]); k2 != kind_bin(A, c)) {
+                    // recycled page: undo, then re-publish it for its real
+                    // owner (as bin_reclaim's ABA path does): a claimer of
+                    // (A', c') may have seen our bits and dropped the page
+                    undo_claim(h, p, i, got, k2);
                     return 0;
                 }
                 if (((old | m) | ~vm) == ~0ull) {                  // this word is full now
@@ -863,7 +873,6 @@ static __device__ GA_CLAIM_FN uint64_t bin_claim_page(const ga_desc* h, uint64_t
             }
             fr = ~(old | m) & vm;
         }
-#endif
     }
     nonfull_clear_if_full(h, p, c, A);
     return 0;
@@ -873,7 +882,7 @@ static __device__ GA_CLAIM_FN uint64_t bin_claim_page(const ga_desc* h, uint64_t
 // Debug builds: a claimer stuck in bin_find_chunk audits arena A's class-c
 // bins once (single auditor) into the debug header words 1..7.
 static __device__ __noinline__ void nfc_audit(const ga_desc* h, uint32_t A, int c) {
-    uint64_t* dbg = g_ga_dbg;
+    uint64_t* dbg = h->dbg;
     if (!dbg || atomicCAS((unsigned long long*)&dbg[1], 0ull, 1ull) != 0ull) return;
     HB3 nb = arena_hb(h, A, kAhbNfc + c);
     uint64_t nbins = 0, nfree = 0, lost_nf = 0, lost_sum = 0, lost_up = 0;
@@ -935,7 +944,7 @@ static __device__ __noinline__ void nfc_repair(const ga_desc* h, uint32_t A, int
             stat_add(h, kStatRepairSummary, 1);
         }
     }
-    if (g_ga_dbg && atomicCAS((unsigned long long*)&g_ga_dbg[1], 0ull, 1ull) == 0ull) {
+    if (h->dbg && atomicCAS((unsigned long long*)&h->dbg[1], 0ull, 1ull) == 0ull) {
         // one diagnostic dump (header words 2..7): where are arena A's class-c
         // units?  Spans / bins of kind (A, c) anywhere, their free slots, how
         // many sit in chunks not owned by A, how many lack their non-full bit.
@@ -961,7 +970,7 @@ static __device__ __noinline__ void nfc_repair(const ga_desc* h, uint32_t A, int
             else if (k != kind_bin(A, c)) owned_other++;
         }
         const uint64_t sw = ld_rlx(sem_ptr(h, A, c));
-        volatile uint64_t* r = (volatile uint64_t*)g_ga_dbg;
+        volatile uint64_t* r = (volatile uint64_t*)h->dbg;
         r[2] = ((uint64_t)A << 8) | (uint64_t)c | ((uint64_t)(uint32_t)sem_C(sw) << 32);
         r[3] = nb_all; r[4] = free_all; r[5] = foreign | (free_foreign << 32); r[6] = nf_missing;
         r[7] = ((uint64_t)(uint32_t)sem_D(sw) << 32);
@@ -1098,14 +1107,16 @@ static __device__ __noinline__ bool bin_reclaim(const ga_desc* h, uint64_t p, ui
 
 
 // Reclaim up to `budget` candidate bins of arena A (budget < 0: all), leaving
-// at least `keep` free slots per class (0: reclaim every empty bin).
-static __device__ __noinline__ void reclaim_arena(const ga_desc* h, uint32_t A, int budget, uint32_t keep) {
+// at least `keep` free slots per class (0: reclaim every empty bin).  Returns
+// the number of bins reclaimed.
+static __device__ __noinline__ int reclaim_arena(const ga_desc* h, uint32_t A, int budget, uint32_t keep) {
     HB3 cb = arena_hb(h, A, kAhbCnd);
-    if (!hb3_any(cb)) return;
+    if (!hb3_any(cb)) return 0;
     uint32_t seed = scatter_seed();
+    int done = 0;
     while (budget != 0) {
         int64_t j = hb3_find(cb, seed);
-        if (j < 0) return;
+        if (j < 0) return done;
         uint64_t cm = ld_rlx(&cb.w0[j]);
         if (!cm) { hb3_up_clear(cb, (uint32_t)j); continue; }
         uint64_t ch = (uint64_t)j * 64 + (uint64_t)(__ffsll((long long)cm) - 1);
@@ -1116,7 +1127,8 @@ static __device__ __noinline__ void reclaim_arena(const ga_desc* h, uint32_t A, 
             uint32_t pb = (uint32_t)(__ffsll((long long)pm) - 1);
             pm &= pm - 1;
             if (budget == 0) { mark_candidate(h, ch * kChunkPages + pb, A); continue; }
-            if (!bin_reclaim(h, ch * kChunkPages + pb, keep)) {
+            if (bin_reclaim(h, ch * kChunkPages + pb, keep)) done++;
+            else {
                 // still empty but the class needs it for now: keep it a candidate
                 uint64_t w[4];
                 ld_bitmap(page_bits(h, ch * kChunkPages + pb), w);
@@ -1132,9 +1144,10 @@ static __device__ __noinline__ void reclaim_arena(const ga_desc* h, uint32_t A, 
         }
         if (pm_left) {                                      // re-mark what could not go yet
             summarised_set(cb, ch, &h->chunk_cand[ch], pm_left);
-            return;                                         // and stop: the rest is in use too
+            return done;                                    // and stop: the rest is in use too
         }
     }
+    return done;
 }
 static __device__ __noinline__ void reclaim_all(const ga_desc* h) {
     for (uint32_t A = 0; A < h->n_arenas; A++) reclaim_arena(h, A, -1, 0);
@@ -1331,7 +1344,7 @@ static __device__ __noinline__ uint64_t bin_claim_collective(const ga_desc* h, u
                    __reduce_or_sync(unsat, (uint32_t)drop));
         }
 #endif
-        unsat = __ballot_sync(unsat, my == kNull);
+        unsat = opaque_mask(__ballot_sync(unsat, my == kNull));
         if (my != kNull) break;                             // a satisfied lane leaves the group
     }
     return my;
@@ -1393,7 +1406,7 @@ static __device__ __noinline__ uint64_t bin_grow_collective(const ga_desc* h, un
         pages_left -= np;
         mode = 0;
     }
-    __syncwarp(grp);
+    warp_release(grp);
     if ((int)lane == leader) {
         stat_add(h, kStatBinGrow, k);
         st_rlx32(&h->hint[A * kNcls + c], (uint32_t)last_page);
@@ -1434,7 +1447,7 @@ static __device__ __noinline__ uint64_t span_grow_collective(const ga_desc* h, u
         }
         served += take;
     }
-    __syncwarp(grp);
+    warp_release(grp);
     if ((int)lane == leader) {
         stat_add(h, kStatBinGrow, (served + slots - 1) / slots);
         if (ch >= 0) {
@@ -1482,6 +1495,7 @@ static __device__ __noinline__ uint64_t tree_malloc_group(const ga_desc* h, unsi
     }
     m = __shfl_sync(grp, m, leader);
     if (m < 0) return kNull;
+    if ((int)lane == leader) reserve_add(h, (int64_t)N << o);
     Nm = __shfl_sync(grp, Nm, leader);
     const int s = m - o;
     uint64_t my = kNull;
@@ -1517,12 +1531,20 @@ static __device__ __noinline__ uint64_t tree_malloc_group(const ga_desc* h, unsi
         }
         served += cap < N - served ? cap : N - served;
     }
+    // Every right part is published before any lane returns its block: a lane
+    // that frees its block at once must find the split's other halves already
+    // Available, or its merge (tree_free's CAS on the sibling word, R-21) would
+    // mark it Available beside a buddy published a moment later -- two
+    // Available siblings (found by tests/test_gpu_edge.py on the GA_NSPAN=0 build).
+    warp_release(grp);
     return my;
 }
 
 // ---- the entry points ---------------------------------------------------------
+static __device__ __forceinline__ uint64_t* arena_ctr(const ga_desc* h, int i) { return h->actr + arena_of(h) * kActrStride + i; }
 static __device__ __noinline__ uint64_t ga_malloc_off(const ga_desc* h, uint64_t n) {
-    const unsigned act = __activemask();
+    const unsigned act = active_lanes();
+    if ((int)lane_id() == __ffs(act) - 1) red_rlx(arena_ctr(h, 0), __popc(act));    // n_malloc, per warp
     const int key = size_key(h, n);
     const unsigned grp = __match_any_sync(act, key);
     if (key < 0) return kNull;
@@ -1532,25 +1554,13 @@ static __device__ __noinline__ uint64_t ga_malloc_off(const ga_desc* h, uint64_t
         const uint32_t N = __popc(grp), slots = slots_of(key);
         const int leader = __ffs(grp) - 1;
         int r = 0;
-        if ((int)lane_id() == leader)
-        {
+        if ((int)lane_id() == leader) {
+            // the fast acquire inline (one fetch-add, no load gate: the units are
+            // usually there); the exact CAS loop out of line
             uint64_t* sp = sem_ptr(h, A, key);
-#if GA_INL_WAIT
-            // inline fast path: the units are there -> one fetch-add decides
-            const uint64_t dn = (uint64_t)N << 32;
-            r = kBlocked;
-#if GA_FAST_FA
-            {
-#else
-            if (sem_C(ld_rlx(sp)) >= (int32_t)N) {
-#endif
-                uint64_t old = a_add(sp, (uint64_t)0 - dn);
-                if (sem_C(old) >= (int32_t)N) r = kAcquired;
-                else a_add(sp, dn);
-            }
-            if (r != kAcquired)
-#endif
-            r = bsem_wait(sp, N, slots * ((N + slots - 1) / slots), ArenaSpin{h, A});
+            uint64_t w;
+            r = bsem_fast_acquire(sp, N, &w) ? kAcquired
+                                             : bsem_wait_cas(sp, N, slots * ((N + slots - 1) / slots), ArenaSpin{h, A}, w);
         }
         r = __shfl_sync(grp, r, leader);
         my = r == kAcquired ? bin_claim_collective(h, grp, A, key)
@@ -1579,14 +1589,15 @@ static __device__ __noinline__ uint64_t ga_malloc_off(const ga_desc* h, uint64_t
 // free), then each surviving block runs the merge-on-free protocol; bin slots
 // are grouped per bitmap word (one atomicAnd) and per (arena, class) (one signal).
 static __device__ __noinline__ void ga_free_off(const ga_desc* h, uint64_t off) {
-    const unsigned act = __activemask();
+    const unsigned act = active_lanes();
     uint32_t k = 0;
     uint64_t p = 0;
     if (off != kNull) { p = off >> kPageShift; k = ld_rlx32(&h->kind[p]); }
     const bool is_bin = (off != kNull) && ((k & 0xC0000000u) == kKindBin);
     const bool is_tree = (off != kNull) && !is_bin;
-    const unsigned bins = __ballot_sync(act, is_bin);
-    const unsigned trees = __ballot_sync(act, is_tree);
+    const unsigned bins = opaque_mask(__ballot_sync(act, is_bin));
+    const unsigned trees = opaque_mask(__ballot_sync(act, is_tree));
+    if ((int)lane_id() == __ffs(act) - 1 && (bins | trees)) red_rlx(arena_ctr(h, 1), __popc(bins | trees));   // n_free
     if (is_tree) {
         int n = (int)(k & 0xFF);                               // order from the page kind (R-18)
         uint64_t x = p >> n;
@@ -1603,7 +1614,7 @@ static __device__ __noinline__ void ga_free_off(const ga_desc* h, uint64_t off) 
                 if ((int)lane_id() == __ffs(mm) - 1) { x >>= 1; n++; }   // both halves are ours: merged
                 else alive = false;
             }
-            part = __ballot_sync(part, alive);
+            part = opaque_mask(__ballot_sync(part, alive));
             if (!alive) break;
         }
         if (alive) tree_free(h, n, x);
@@ -1636,7 +1647,10 @@ static __device__ __noinline__ void ga_free_off(const ga_desc* h, uint64_t off) 
             }
         }
     }
-    __syncwarp(bins);
+    // the match is also the execution barrier: every leader's atomicAnd above
+    // has returned (performed at L2) before any lane of `bins` passes it, so
+    // the units signalled below never precede their slots (no __syncwarp: see
+    // opaque_mask)
     const unsigned g2 = __match_any_sync(bins, (A << 4) | (uint32_t)c);     // class < 16
     if ((int)lane_id() == __ffs(g2) - 1) bsem_signal_after_rmw(sem_ptr(h, A, c), __popc(g2));
     if (eager) {

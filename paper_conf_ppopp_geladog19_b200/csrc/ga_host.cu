@@ -22,6 +22,7 @@ namespace {
 
 constexpr uint64_t kAlign = 256;
 constexpr uint64_t kBaseAlign = 2ull << 20;     // R-31: 2 MiB aligned base
+constexpr int kSnapSpanSlots = 5;               // snapshot format: class entries 4 .. 64 KiB (include/ga.h)
 
 inline uint64_t up(uint64_t x, uint64_t a) { return (x + a - 1) / a * a; }
 inline uint64_t sem_word(int32_t C, int32_t D) { return ((uint64_t)(uint32_t)C << 32) | (uint32_t)(D + 0x80000000u); }
@@ -72,13 +73,13 @@ ga_status init_heap(ga_heap_t h, cudaStream_t s) {
     k_fill_u64<<<grid_for((uint64_t)d.n_arenas * kSemStride), 256, 0, s>>>(d.psem, (uint64_t)d.n_arenas * kSemStride, sem_word(0, 0));
     k_fill_u32<<<grid_for((uint64_t)d.n_arenas * kNcls), 256, 0, s>>>(d.hint, (uint64_t)d.n_arenas * kNcls, 0xFFFFFFFFu);
     k_fill_u64<<<grid_for(h->ahb_total_words), 256, 0, s>>>(d.ahb, h->ahb_total_words, 0ull);
-    k_fill_u64<<<1, 32, 0, s>>>(d.stats, 16, 0ull);
+    k_fill_u64<<<1, 32, 0, s>>>(d.stats, kStatWords, 0ull);
+    k_fill_u64<<<grid_for((uint64_t)d.n_arenas * kActrStride), 256, 0, s>>>(d.actr, (uint64_t)d.n_arenas * kActrStride, 0ull);
     k_fill_u32<<<1, 64, 0, s>>>(d.lvl_hint, 48, 0u);
     if (!chk(cudaGetLastError())) return GA_ECUDA;
     if (!chk(cudaMemcpyAsync(h->ddesc, &h->dev, sizeof(ga_desc), cudaMemcpyHostToDevice, s))) return GA_ECUDA;
     if (!chk(cudaMemcpyAsync(d.avail, h->avail_init.data(), h->avail_words * 8, cudaMemcpyHostToDevice, s))) return GA_ECUDA;
     if (!chk(cudaMemcpyAsync(d.tsem, h->tsem_init.data(), h->tsem_init.size() * 8, cudaMemcpyHostToDevice, s))) return GA_ECUDA;
-    h->peak_reserved_pages = 0;
     return GA_OK;
 }
 
@@ -169,7 +170,8 @@ ga_status ga_heap_create(int device, ga_stream_t stream, void* buf, size_t bytes
     uint64_t o_owned = cv.take<uint64_t>(h->ahb_total_words);
     uint64_t o_avail = cv.take<uint64_t>(aw);
     uint64_t o_tsem = cv.take<uint64_t>((uint64_t)(L + 1) * kSemStride);
-    uint64_t o_stats = cv.take<uint64_t>(16);
+    uint64_t o_stats = cv.take<uint64_t>(kStatWords);
+    uint64_t o_actr = cv.take<uint64_t>((uint64_t)d.n_arenas * kActrStride);
     uint64_t o_lhint = cv.take<uint32_t>(48);
     h->meta_bytes = cv.off;
     if (cudaMalloc(&h->meta, h->meta_bytes) != cudaSuccess) { delete h; cudaSetDevice(prev); return GA_ENOMEM; }
@@ -195,6 +197,7 @@ ga_status ga_heap_create(int device, ga_stream_t stream, void* buf, size_t bytes
     d.avail = (uint64_t*)(m + o_avail);
     d.tsem = (uint64_t*)(m + o_tsem);
     d.stats = (uint64_t*)(m + o_stats);
+    d.actr = (uint64_t*)(m + o_actr);
     d.lvl_hint = (uint32_t*)(m + o_lhint);
     // empty heap: the binary decomposition of the pages into maximal aligned roots (R-30)
     h->avail_init.assign(aw, 0ull);
@@ -232,6 +235,7 @@ ga_status ga_heap_destroy(ga_heap_t h) {
 
 ga_status ga_heap_reset(ga_heap_t h, ga_stream_t stream) {
     if (!h) return GA_EINVAL;
+    DeviceGuard g(h->device);
     return init_heap(h, (cudaStream_t)stream);
 }
 
@@ -252,6 +256,7 @@ ga_status ga_heap_info(ga_heap_t h, uint64_t* heap_bytes, void** base, uint64_t*
 
 ga_status ga_heap_quiesce(ga_heap_t h, ga_stream_t stream) {
     if (!h) return GA_EINVAL;
+    DeviceGuard g(h->device);
     cudaStream_t s = (cudaStream_t)stream;
     k_quiesce_bins<<<grid_for(h->dev.pages), 256, 0, s>>>(h->ddesc);
     k_quiesce_chunks<<<grid_for(h->dev.nchunks), 256, 0, s>>>(h->ddesc);
@@ -262,6 +267,7 @@ ga_status ga_heap_quiesce(ga_heap_t h, ga_stream_t stream) {
 
 ga_status ga_reserved_pages(ga_heap_t h, ga_stream_t stream, uint64_t* out) {
     if (!h || !out) return GA_EINVAL;
+    DeviceGuard g(h->device);
     const ga_desc& d = h->dev;
     std::vector<uint64_t> av(h->avail_words);
     if (cudaMemcpyAsync(av.data(), d.avail, h->avail_words * 8, cudaMemcpyDeviceToHost, (cudaStream_t)stream) != cudaSuccess) return GA_ECUDA;
@@ -273,26 +279,32 @@ ga_status ga_reserved_pages(ga_heap_t h, ga_stream_t stream, uint64_t* out) {
         avail_pages += cnt << n;
     }
     *out = d.pages - avail_pages;
-    if (*out > h->peak_reserved_pages) h->peak_reserved_pages = *out;
     return GA_OK;
 }
 
 ga_status ga_stats(ga_heap_t h, ga_stream_t stream, ga_stats_t* out) {
     if (!h || !out) return GA_EINVAL;
+    DeviceGuard g(h->device);
     memset(out, 0, sizeof *out);
-    uint64_t st[16];
-    if (cudaMemcpyAsync(st, h->dev.stats, sizeof st, cudaMemcpyDeviceToHost, (cudaStream_t)stream) != cudaSuccess) return GA_ECUDA;
-    uint64_t res = 0;
-    ga_status r = ga_reserved_pages(h, stream, &res);
-    if (r != GA_OK) return r;
-    std::vector<uint64_t> cand(h->dev.nchunks);
-    if (cudaMemcpy(cand.data(), h->dev.chunk_cand, h->dev.nchunks * 8, cudaMemcpyDeviceToHost) != cudaSuccess) return GA_ECUDA;
+    const ga_desc& d = h->dev;
+    cudaStream_t s = (cudaStream_t)stream;
+    uint64_t st[kStatWords];
+    std::vector<uint64_t> ctr((uint64_t)d.n_arenas * kActrStride), cand(d.nchunks);
+    bool ok = cudaMemcpyAsync(st, d.stats, sizeof st, cudaMemcpyDeviceToHost, s) == cudaSuccess &&
+              cudaMemcpyAsync(ctr.data(), d.actr, ctr.size() * 8, cudaMemcpyDeviceToHost, s) == cudaSuccess &&
+              cudaMemcpyAsync(cand.data(), d.chunk_cand, cand.size() * 8, cudaMemcpyDeviceToHost, s) == cudaSuccess &&
+              cudaStreamSynchronize(s) == cudaSuccess;
+    if (!ok) return GA_ECUDA;
     uint64_t pend = 0;
     for (uint64_t c : cand) pend += (uint64_t)__builtin_popcountll(c);
-    out->heap_bytes = h->dev.pages * kPage;
+    for (uint32_t A = 0; A < d.n_arenas; A++) {
+        out->n_malloc += ctr[(uint64_t)A * kActrStride + 0];
+        out->n_free += ctr[(uint64_t)A * kActrStride + 1];
+    }
+    out->heap_bytes = d.pages * kPage;
     out->metadata_bytes = h->meta_bytes;
-    out->reserved_bytes = res * kPage;
-    out->peak_reserved_bytes = h->peak_reserved_pages * kPage;
+    out->reserved_bytes = st[kStatReserved] * kPage;
+    out->peak_reserved_bytes = st[kStatPeakReserved] * kPage;
     out->n_bin_grow = st[kStatBinGrow];
     out->n_chunk_grow = st[kStatChunkGrow];
     out->n_bin_reclaim = st[kStatBinReclaim];
@@ -302,12 +314,14 @@ ga_status ga_stats(ga_heap_t h, ga_stream_t stream, ga_stats_t* out) {
     out->n_pending_reclaim = pend;
     out->n_repair_nonfull = st[kStatRepairNonfull];
     out->n_repair_summary = st[kStatRepairSummary];
-    out->n_arenas = h->dev.n_arenas;
+    out->n_waiter_reclaim = st[kStatWaiterReclaim];
+    out->n_arenas = d.n_arenas;
     return GA_OK;
 }
 
 ga_status ga_heap_snapshot(ga_heap_t h, ga_stream_t stream, void* host, size_t cap, size_t* used) {
     if (!h || !used) return GA_EINVAL;
+    DeviceGuard g(h->device);
     const ga_desc& d = h->dev;
     cudaStream_t s = (cudaStream_t)stream;
     std::vector<uint64_t> bits(d.pages * kBinWords), used_(d.nchunks), nonfull(1), cand(d.nchunks);
@@ -332,7 +346,9 @@ ga_status ga_heap_snapshot(ga_heap_t h, ga_stream_t stream, void* host, size_t c
     put64(d.pages * kPage);
     put64(d.pages);
     put64(kPage | ((uint64_t)(d.L + 1) << 32));
-    put64((1ull << kMinShift) | ((uint64_t)kNbin << 32) | ((uint64_t)kNspan << 40) | ((uint64_t)kChunkPages << 48));
+    // the format's class section covers 16 B .. 64 KiB whatever this build
+    // routes to spans (kSnapSpanSlots entries above the bins; zeros past kNspan)
+    put64((1ull << kMinShift) | ((uint64_t)kNbin << 32) | ((uint64_t)kSnapSpanSlots << 40) | ((uint64_t)kChunkPages << 48));
     std::vector<uint8_t> kb(d.pages, 0x00);
     for (uint32_t n = 0; n <= d.L; n++) {
         uint64_t cnt = 1ull << (d.L - n);
@@ -371,8 +387,9 @@ ga_status ga_heap_snapshot(ga_heap_t h, ga_stream_t stream, void* host, size_t c
         uint64_t cnt = 1ull << (d.L - n), nb = (cnt + 7) / 8;
         put(&av[d.lvl_off[n]], nb);                         // little endian words == LSB-first bytes
     }
-    for (int c = 0; c < kNcls; c++) {
+    for (int c = 0; c < kNbin + kSnapSpanSlots; c++) {
         int64_t sc = 0, md = 0;
+        if (c >= kNcls) { put64(0); put64(0); continue; }
         for (uint32_t A = 0; A < d.n_arenas; A++) {
             uint64_t w = sem[((uint64_t)A * kNcls + c) * kSemStride];
             int32_t C = (int32_t)(uint32_t)(w >> 32), D = (int32_t)((uint32_t)w - 0x80000000u);

@@ -4,6 +4,8 @@
 #include <cstdint>
 #include <vector>
 
+#include <cuda_runtime.h>
+
 #include "ga.h"
 
 struct ga_heap_s {
@@ -17,7 +19,19 @@ struct ga_heap_s {
     std::vector<uint64_t> tsem_init;
     uint64_t avail_words = 0;
     uint64_t ahb_total_words = 0;
-    uint64_t peak_reserved_pages = 0;
     void* scratch = nullptr;       // device scratch for ga_trace_timed_host
     size_t scratch_bytes = 0;
+};
+
+// Handle-taking host calls run on the heap's device and restore the caller's
+// current device on return.
+struct DeviceGuard {
+    int prev = -1;
+    explicit DeviceGuard(int dev) {
+        if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+        else if (prev != dev) cudaSetDevice(dev);
+    }
+    ~DeviceGuard() { if (prev >= 0) cudaSetDevice(prev); }
+    DeviceGuard(const DeviceGuard&) = delete;
+    DeviceGuard& operator=(const DeviceGuard&) = delete;
 };

@@ -62,7 +62,8 @@ class TraceRun:
     counts: dict
     log: np.ndarray | None = None
     peak_reserved_bytes: int = 0
-    reserved_per_round: list = field(default_factory=list)
+    reserved_per_round: list = field(default_factory=list)        # from the tree bitmaps (ga_reserved_pages)
+    reserved_dev_per_round: list = field(default_factory=list)    # the device counter (ga_stats)
     live_per_round: list = field(default_factory=list)   # requested bytes held at each boundary
 
     @property
@@ -103,6 +104,7 @@ def run_correctness(heap: GpuHeap | None, sizes: np.ndarray, D: int, log: bool =
                                     flags, block)
             if heap and reserved and r < R:
                 run.reserved_per_round.append(heap.reserved_bytes())
+                run.reserved_dev_per_round.append(heap.stats()["reserved_bytes"])
                 run.live_per_round.append(int(held[1::2].sum().item()))
         else:
             for ph in (0, 1):
@@ -114,6 +116,7 @@ def run_correctness(heap: GpuHeap | None, sizes: np.ndarray, D: int, log: bool =
                                         flags, block)
                 if heap and reserved and ph == 0:
                     run.reserved_per_round.append(heap.reserved_bytes())
+                    run.reserved_dev_per_round.append(heap.stats()["reserved_bytes"])
                     run.live_per_round.append(int(held[1::2].sum().item()))
     st.synchronize()
     run.counts = _counts(counts)

@@ -11,6 +11,8 @@ placements are correct -- only what is unique:
 * quiescent GPU snapshots satisfy the oracle's invariants (semaphore counts ==
   free resources, buddy properties).
 """
+import os
+
 import numpy as np
 import pytest
 import torch
@@ -32,7 +34,17 @@ def _cuda():
     torch.cuda.set_device(0)
 
 
+def test_loaded_build():
+    """The library under test is the one the run asked for (GA_LIB variants,
+    tests/test_gpu_variants.py): its span classes match GA_EXPECT_NSPAN."""
+    want = os.environ.get("GA_EXPECT_NSPAN")
+    lay = ga.ga_layout()
+    assert lay["n_span_classes"] == (int(want) if want is not None else 5)
+
+
 def _empty_parity(heap: GpuHeap):
+    st = heap.stats()                                   # the safety net never ran (ga.h: expected 0)
+    assert st["n_repair_nonfull"] == 0 and st["n_repair_summary"] == 0, st
     heap.quiesce()
     snap = heap.snapshot()
     errs = S.check(S.parse(snap), require_reclaimed=True)

@@ -130,3 +130,77 @@ def test_group_demand_can_overproduce():
     res = explore([5, 1, 1], 4, 4)
     used = {u for _, u, _ in res["terminals"]}
     assert used >= {2} and max(used) <= 3
+
+
+# ---------------------------------------------------------------------------
+# The CUDA path's own semaphore protocols (oracle/bsem.py explore_gpu), checked
+# against Alg. 1 on every interleaving of their atomic steps.
+# ---------------------------------------------------------------------------
+from oracle.bsem import explore_gpu  # noqa: E402
+
+
+@pytest.mark.parametrize("form", ["arena", "tree"])
+def test_gpu_forms_unit_demand_exact(form):
+    """T <= 6 threads of demand 1 (the Fig. 5 setting): the forms
+    the CUDA path runs grant exactly min(T, pool*B) units (no false starvation,
+    P:L488-506), use exactly min(pool, ceil(T/B)) batches (no over-production),
+    never deadlock, never over-grant, end with D = 0, and are conservative in
+    every reachable state (R-35)."""
+    for T in range(1, 7):
+        for B in (2, 3, 4):
+            for pool in range(0, 4):
+                r = explore_gpu([1] * T, B, pool, form)
+                assert r["deadlocks"] == 0 and r["nonconservative"] == 0 and r["overgrant"] == 0, (T, B, pool)
+                for (C, D), used, res in r["terminals"]:
+                    ok = sum(o for _, o in res)
+                    assert ok == min(T, pool * B), (T, B, pool, res)
+                    assert used == min(pool, -(-T // B)), (T, B, pool, used)
+                    assert D == 0 and C == used * B - ok
+
+
+def _mixed_cases():
+    import itertools
+    for release in (False, True):
+        for n in (2, 3):
+            for Ns in itertools.combinations_with_replacement([1, 2, 3, 4], n):
+                for B in (2, 4):
+                    for C0 in (0, 1, 3, 4):
+                        for pool in (1, 2, 3):
+                            yield release, Ns, B, C0, pool
+
+
+def test_gpu_forms_mixed_group_demand():
+    """Warp groups (demand N > 1, reading R-8): on every interleaving the forms
+    never deadlock, never over-grant, stay conservative, end with D = 0 and
+    C = C0 + produced - held; they use at most ONE batch more than Alg. 1's
+    worst interleaving (the over-production bound recorded in DESIGN.md R-35).
+    Round 1's forms are checked too: they are not conservative."""
+    worst = {"arena": 0, "tree": 0}
+    for release, Ns, B, C0, pool in _mixed_cases():
+        ref = explore_gpu(Ns, B, pool, "alg1", release=release, init_C=C0)
+        ref_max = max(u for _, u, _ in ref["terminals"])
+        for form in ("arena", "tree"):
+            r = explore_gpu(Ns, B, pool, form, release=release, init_C=C0)
+            assert r["deadlocks"] == 0 and r["nonconservative"] == 0 and r["overgrant"] == 0
+            for (C, D), used, res in r["terminals"]:
+                held = 0 if release else sum(N for N, o in res if o)
+                assert D == 0 and C == C0 + used * B - held, (form, Ns, B, C0, pool, res)
+            worst[form] = max(worst[form], max(u for _, u, _ in r["terminals"]) - ref_max)
+    assert worst == {"arena": 1, "tree": 1}, worst
+
+
+def test_round1_forms_are_caught():
+    """Sensitivity of the checker: round 1's fast paths are flagged.
+    * the unconditional fetch-add C -= N hid units from other deciders: states
+      are not conservative, and a warp group fails while a batch is left that
+      Alg. 1 would have used (P:L488-506);
+    * the optimistic TBuddy form starves a unit-demand thread (Alg. 1 never does)."""
+    r = explore_gpu([1, 3], 2, 2, "arena_old", init_C=1)
+    ref = explore_gpu([1, 3], 2, 2, "alg1", init_C=1)
+    assert r["nonconservative"] > 0
+    outcomes = {(u, res) for _, u, res in r["terminals"]}
+    assert outcomes - {(u, res) for _, u, res in ref["terminals"]}
+    assert any(not all(o for _, o in res) and u < 2 for u, res in outcomes)
+    r = explore_gpu([1, 1], 2, 1, "tree_old")
+    assert any(sum(o for _, o in res) < 2 for _, _, res in r["terminals"])
+    assert r["nonconservative"] > 0
