@@ -358,3 +358,63 @@ def test_snapshot_checker_catches_broken_states():
     s = S.parse(bytes(buf))
     s.kind[3] = S.K_FREE_INTERIOR
     assert S.check(s)
+
+
+def _paper_fill(heap_bytes, sizes_cycle, seed):
+    """Fill a paper-layout oracle heap with requests drawn from sizes_cycle
+    until every size fails; returns [(offset, class_bytes)]."""
+    h = oracle.Heap(heap_bytes, PAPER)
+    rng = np.random.default_rng(seed)
+    live, alive = [], set(sizes_cycle)
+    while alive:
+        n = int(rng.choice(sorted(alive)))
+        off = h.malloc(n)
+        if off is None:
+            alive.discard(n)
+            continue
+        live.append((off, max(8, 1 << (n - 1).bit_length())))
+    return h, live
+
+
+@pytest.mark.parametrize("sizes", [(8, 16, 32, 64, 128), (8, 128), (16, 32, 256, 512, 1024), (8, 64, 1024, 2048, 4096)])
+def test_paper_layout_slots_disjoint_and_outside_headers(sizes):
+    """Reading R-11 (paper layout): every chunk keeps 128 B
+    in-band headers at the start of each of its 64 pages (chunk header, the 62
+    bin headers, the second header bin), bin bodies start at +128, and the 62
+    128-byte tails live in the two header pages (tail t at chunk offset
+    128 + 128t for t < 31, else 4096 + 128 + 128(t - 31)).  At full fill with
+    mixed classes -- so every bin of every chunk uses its tail -- the slots are
+    pairwise disjoint, aligned to min(class, 128) relative to their page, inside
+    the heap, and none touches a header.  A tail off by one slot (or placed in
+    the wrong header page) overlaps a neighbour or a header and fails here.
+    Freeing everything restores the fresh heap."""
+    heap_bytes = 4 * 256 << 10
+    h, live = _paper_fill(heap_bytes, sizes, seed=len(sizes) * 7 + sizes[0])
+    offs = np.array([o for o, _ in live], dtype=np.int64)
+    lens = np.array([c for _, c in live], dtype=np.int64)
+    assert offs.min() >= 0 and (offs + lens).max() <= heap_bytes
+    idx = np.argsort(offs)
+    assert np.all(offs[idx][1:] >= offs[idx][:-1] + lens[idx][:-1]), "overlapping slots"
+    bins = lens <= 1024                                   # UAlloc slots (2 KB goes to a 4 KB page)
+    in_page = offs[bins] % 4096
+    assert np.all((in_page >= 128) | (lens[bins] > 4096)), "a slot inside a 128 B header"
+    assert np.all((in_page % np.minimum(lens[bins], 128)) == 0)
+    if 8 in sizes and 128 in sizes:                       # tails used: slots in pages 0/1 of chunks
+        pg = (offs[bins] // 4096) % 64
+        assert np.any(pg == 0) and np.any(pg == 1)
+    fresh = oracle.snapshot_of_fresh(heap_bytes, PAPER)
+    for o, _ in live:
+        assert h.free(o) == 0
+    assert h.snapshot() == fresh
+    h.close()
+
+
+def test_paper_layout_tail_capacity_per_chunk():
+    """One chunk filled with 128 B requests: 62 bins x (3968/128 body slots + 1
+    tail slot) = 62 x 32 = 1984 slots; the tails supply exactly
+    62 of them, all inside the two header pages."""
+    h, live = _paper_fill(256 << 10, (128,), seed=1)
+    assert len(live) == 62 * 32
+    pg = np.array([(o // 4096) % 64 for o, _ in live])
+    assert int((pg <= 1).sum()) == 62
+    h.close()
