@@ -205,18 +205,25 @@ def run_reference(args, trace):
 def config_of(trace, args):
     return {"workload": trace.name, "threads": trace.T, "rounds": trace.R, "free_depth": trace.D,
             "heap_bytes": trace.heap_bytes, "sizes": "n = 2^k + U[1,2^k], k~U{3..15} (16 B - 64 KiB classes)",
-            "block": args.block, "l2": "flushed between steps (512 MiB write)", "seed": hex(trace.seed)}
+            "block": args.block, "l2": "flushed between steps (512 MiB write)", "heap_state": "cold (reset per step)",
+            "seed": hex(trace.seed)}
 
 
 def d3_sweep(ga, heap, stream, dev, T, args, sizes=(16, 32, 64, 128, 256, 512, 1024, 2048, 4096, 8192), R=16):
+    """d3 (BASELINE configs[2]): warp-uniform size s, every thread R rounds of
+    malloc(s) + free on a 4 GiB heap at full occupancy, heap reset (untimed)
+    before every rep; CUDA malloc on one round of the same trace; fragmentation
+    of one malloc-only phase (correctness mode) beside the oracle's."""
     import torch
+    import oracle
+    from paper_conf_ppopp_geladog19_b200.runner import run_correctness
     res = {}
     cc = torch.zeros(8, dtype=torch.int64, device=dev)
     for sz in sizes:
         d = torch.full((R * T,), sz, dtype=torch.int32, device=dev)
-        heap.reset()
-        times = []
+        times, fails = [], 0
         for rep in range(4):
+            heap.reset()
             cc.zero_()
             a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             a0.record(stream)
@@ -225,9 +232,9 @@ def d3_sweep(ga, heap, stream, dev, T, args, sizes=(16, 32, 64, 128, 256, 512, 1
             a1.synchronize()
             if rep:
                 times.append(a0.elapsed_time(a1) / 1e3)
-        c = cc.cpu().numpy()
-        ours = float(c[0] + c[2]) / (sum(times) / len(times))
-        fails = int(c[1])
+                fails += int(cc[1].item())
+        times.sort()
+        ours = float(R * T * 2) / times[len(times) // 2]
         cc.zero_()
         a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a0.record(stream)
@@ -236,21 +243,29 @@ def d3_sweep(ga, heap, stream, dev, T, args, sizes=(16, 32, 64, 128, 256, 512, 1
         a1.synchronize()
         c = cc.cpu().numpy()
         cuda = float(c[0] + c[2]) / (a0.elapsed_time(a1) / 1e3)
-        res[str(sz)] = {"ours": ours, "cuda_malloc": cuda, "speedup": ours / cuda, "ours_failed": fails,
-                        "cuda_failed": int(c[1]), "ours_rounds": R, "cuda_rounds": 1}
-    vals = [v["speedup"] for v in res.values()]
-    res["min_speedup"] = min(vals)
-    res["geomean_speedup"] = float(np.exp(np.mean(np.log(vals))))
+        one = np.full((1, T), sz, dtype=np.uint32)
+        heap.reset()
+        run = run_correctness(heap, one, 0, log=False, tag=False, reserved=True)
+        ref = oracle.run_trace(one, heap.heap_bytes, 0, want_ok=False).stats
+        fg = run.peak_reserved_bytes / run.peak_live_bytes
+        fo = ref["peak_reserved_bytes"] / ref["peak_live_bytes"]
+        res[str(sz)] = {"Gcalls_s": ours / 1e9, "cuda_Mcalls_s": cuda / 1e6, "x_cuda": ours / cuda,
+                        "failed": fails + int(c[1]) + run.counts["n_fail"],
+                        "frag": {"gpu": round(fg, 4), "oracle": round(fo, 4), "ratio": round(fg / fo, 4)}}
+    vals = [v["x_cuda"] for v in res.values()]
+    res["min_x_cuda"] = min(vals)
+    res["geomean_x_cuda"] = float(np.exp(np.mean(np.log(vals))))
+    res["max_frag_ratio"] = max(v["frag"]["ratio"] for k, v in res.items() if isinstance(v, dict))
     return res
 
 
 def d4_levels(ga, stream, dev, args, flush, levels=("fit", "exhaust", "overcommit"), reps=3):
-    """d4 at the other two pressure levels: the same mixed trace on
+    """d4 at the other pressure levels: the same mixed trace on
     a 16 GiB heap (fit: every malloc succeeds), a 3 GiB heap (exhaust: the peak
     reserved reaches ~99 % of the heap) and a 2.75 GiB heap (overcommit: below
-    the oracle's own peak reserved, so both sides fail mallocs and reclaim under
-    real exhaustion).  calls/s from the timed
-    kernel; failures and fragmentation from correctness mode, beside the oracle's."""
+    the oracle's own peak reserved, so both sides fail mallocs).  calls/s from
+    the timed kernel on a cold heap; failures and fragmentation from correctness
+    mode, beside the oracle's."""
     import torch
     import oracle
     from paper_conf_ppopp_geladog19_b200.runner import GpuHeap, run_correctness
@@ -263,6 +278,7 @@ def d4_levels(ga, stream, dev, args, flush, levels=("fit", "exhaust", "overcommi
         d = torch.from_numpy(t.sizes.view(np.int32)).to(dev)
         times, fails = [], 0
         for rep in range(reps + 1):
+            heap.reset()
             flush.fill_(rep)
             cc.zero_()
             a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -276,24 +292,26 @@ def d4_levels(ga, stream, dev, args, flush, levels=("fit", "exhaust", "overcommi
         calls = int(cc[0].item() + cc[2].item())
         heap.reset()
         run = run_correctness(heap, t.sizes, t.D, log=False, tag=False, reserved=True)
+        st = heap.stats()
         ref = oracle.run_trace(t.sizes, t.heap_bytes, t.D, want_ok=False).stats
         fg = run.peak_reserved_bytes / run.peak_live_bytes if run.peak_live_bytes else None
         fo = ref["peak_reserved_bytes"] / ref["peak_live_bytes"]
-        st = heap.stats()
-        res[lv] = {"heap_bytes": t.heap_bytes, "calls_per_s": calls / (sum(times) / len(times)),
-                   "ms": 1e3 * sum(times) / len(times), "timed_failed_mallocs": fails,
-                   "correctness_failed_mallocs": run.counts["n_fail"], "oracle_failed_mallocs": ref["n_malloc_fail"],
-                   "fragmentation": {"gpu": fg, "oracle": fo, "ratio": fg / fo if fg else None},
-                   "stats": {k: int(v) for k, v in st.items() if isinstance(v, (int, np.integer))}}
+        res[lv] = {"heap_GiB": t.heap_bytes / 2 ** 30, "ms": 1e3 * sum(times) / len(times),
+                   "Gcalls_s": calls / (sum(times) / len(times)) / 1e9, "failed_timed": fails,
+                   "failed": {"gpu": run.counts["n_fail"], "oracle": ref["n_malloc_fail"]},
+                   "frag": {"gpu": fg, "oracle": fo, "ratio": fg / fo if fg else None},
+                   "reclaims": {"bins": int(st["n_bin_reclaim"]), "by_waiters": int(st["n_waiter_reclaim"])}}
         heap.close()
         del d
     return res
 
 
 def d2_bsem(ga, stream, dev, grid=148 * 8, block=256, iters=32):
-    """wait(k)/signal(k) per thread per iteration on a full grid; ops = wait+signal pairs."""
+    """A summary of d2 (the full k x B x variant matrix is tools/d2_matrix.py):
+    wait(k)/signal(k) per thread per iteration on a full grid, B = 512 (the
+    paper's); G wait+signal pairs per second."""
     import torch
-    names = {0: "warp_aggregated_bulk", 1: "per_thread_bulk", 2: "per_thread_counting", 3: "plain_atomics"}
+    names = {0: "warp_bulk", 1: "thread_bulk", 2: "thread_counting", 3: "plain_atomics"}
     res = {}
     sems = torch.zeros(148 * 4 + 8, dtype=torch.int64, device=dev)
     out = torch.zeros(8, dtype=torch.int64, device=dev)
@@ -302,8 +320,8 @@ def d2_bsem(ga, stream, dev, grid=148 * 8, block=256, iters=32):
             for v in (0, 1, 2, 3):
                 if v == 2 and k != 1:
                     continue
-                cfg = ga.BsemCfg(variant=v, k=k, B=512, n_sems=n_sems, iters=iters, acquire_only=0, grid=grid,
-                                 block=block, seed=tracegen.BASE_SEED + 2)
+                cfg = ga.BsemCfg(variant=v, k=k, B=512, n_sems=n_sems, iters=iters if v != 2 else 4,
+                                 acquire_only=0, grid=grid, block=block, seed=tracegen.BASE_SEED + 2)
                 best = None
                 for rep in range(3):
                     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -314,9 +332,10 @@ def d2_bsem(ga, stream, dev, grid=148 * 8, block=256, iters=32):
                     t = e0.elapsed_time(e1) / 1e3
                     best = t if best is None else min(best, t)
                 o = out.cpu().numpy()
-                res[f"{names[v]}/k={k or 'rand'}/sems={n_sems}"] = {
-                    "pairs_per_s": grid * block * iters / best, "units_per_s": float(o[0]) / best,
-                    "quiescent_C_equals_produced": bool(o[4] == o[3]), "max_abs_D": int(o[5])}
+                ok = bool(o[4] == o[3]) and int(o[5]) == 0
+                res[f"{names[v]}/k={k or 'rand'}/sems={n_sems}"] = round(grid * block * cfg.iters / best / 1e9, 4) \
+                    if ok else "accounting mismatch"
+    res["unit"] = "G wait+signal pairs/s"
     return res
 
 
@@ -341,8 +360,29 @@ def reduce_over_ranks(dist, ms: float, calls: float, device):
     return float(t.item()), float(c.item())
 
 
-# ----------------------------------------------------------------------------- our arm
-def main():
+def launch_or_refuse(args, argv) -> int | None:
+    """--gpus N: one process per GPU.  Without a torchrun environment and N > 1,
+    relaunch this command under torch.distributed.run on N local GPUs; inside
+    one, refuse a WORLD_SIZE that is not N (a silent 1-GPU run would mislabel
+    n_gpus).  None = go on in this process."""
+    world = os.environ.get("WORLD_SIZE")
+    if world is None:
+        if args.gpus <= 1:
+            return None
+        import socket
+        with socket.socket() as so:
+            so.bind(("127.0.0.1", 0))
+            port = so.getsockname()[1]
+        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+               "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__), *argv]
+        return subprocess.call(cmd)
+    if int(world) != args.gpus:
+        sys.stderr.write(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world}; refusing\n")
+        return 2
+    return None
+
+
+def parse_args(argv):
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=10)
@@ -351,175 +391,126 @@ def main():
     ap.add_argument("--block", type=int, default=256)
     ap.add_argument("--no-extras", action="store_true", help="skip CUDA-malloc, sweep, frag, cpu legs")
     ap.add_argument("--cuda-budget-s", type=float, default=20.0)
-    args = ap.parse_args()
+    args = ap.parse_args(argv)
     args.warmup = max(args.warmup, 3)
+    return args
 
-    trace = tracegen.d4_mixed("pressure")
-    if args.impl == "reference":
-        return run_reference(args, trace)
 
-    import torch
-    import paper_conf_ppopp_geladog19_b200 as ga
-    from paper_conf_ppopp_geladog19_b200.runner import GpuHeap, run_correctness
+# ----------------------------------------------------------------------------- our arm (one rank, one GPU)
+class GpuArm:
+    """The device work of one rank: its own heap and trace (replicas), W warm-up
+    and K timed steps of the d4 trace in ONE kernel each, CUDA events on the
+    heap's stream, the heap reset (one kernel, untimed) and L2 flushed before
+    every step; then the same through the C ABI with host buffers (e2e)."""
+    backend = "nccl"
 
-    world = int(os.environ.get("WORLD_SIZE", "1"))
-    rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
-    torch.cuda.set_device(local)
-    dist = None
-    if world > 1:
-        import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    dev = torch.device("cuda", local)
-    stream = torch.cuda.current_stream(dev)
+    def __init__(self, args, rank, local):
+        import torch
+        import paper_conf_ppopp_geladog19_b200 as ga
+        from paper_conf_ppopp_geladog19_b200.runner import GpuHeap
+        self.torch, self.ga, self.args, self.rank = torch, ga, args, rank
+        torch.cuda.set_device(local)
+        self.dev = torch.device("cuda", local)
+        self.reduce_device = self.dev
+        self.local = local
+        self.stream = torch.cuda.current_stream(self.dev)
+        self.trace = rank_trace(tracegen.d4_mixed("pressure"), rank)
+        if not args.no_extras:
+            ga.ga_cuda_set_heap_limit(self.trace.heap_bytes)   # before any kernel that uses malloc
+        self.heap = GpuHeap(self.trace.heap_bytes, device=local, stream=self.stream)
+        self.d_sizes = torch.from_numpy(self.trace.sizes.view(np.int32)).to(self.dev)
+        self.counts = torch.zeros(8, dtype=torch.int64, device=self.dev)
+        self.flush = torch.empty(L2_FLUSH_BYTES // 4, dtype=torch.int32, device=self.dev)
 
-    # per-rank trace (replicas: seed + rank); rank 0 uses the canonical trace
-    trace = rank_trace(trace, rank)
-    R, T, D = trace.R, trace.T, trace.D
-    if not args.no_extras:
-        ga.ga_cuda_set_heap_limit(trace.heap_bytes)       # before any kernel that uses malloc
-    heap = GpuHeap(trace.heap_bytes, device=local, stream=stream)
-    d_sizes = torch.from_numpy(trace.sizes.view(np.int32)).to(dev)
-    counts = torch.zeros(8, dtype=torch.int64, device=dev)
-    flush = torch.empty(L2_FLUSH_BYTES // 4, dtype=torch.int32, device=dev)
+    def _step(self):
+        t = self.trace
+        self.ga.ga_trace_timed(self.heap.h, self.stream.cuda_stream, self.d_sizes.data_ptr(), t.R, t.T, t.D,
+                               self.counts.data_ptr(), self.args.block)
 
-    def step():
-        ga.ga_trace_timed(heap.h, stream.cuda_stream, d_sizes.data_ptr(), R, T, D, counts.data_ptr(), args.block)
-
-    def timed_steps(n, cold):
-        """n steps, each bracketed by CUDA events on the heap's stream.  cold: the
-        heap is reset (ga_heap_reset, untimed) before every step, SURVEY 8(d)."""
+    def _timed_steps(self, n, cold):
+        torch = self.torch
         ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(n)]
         for i, (s, e) in enumerate(ev):
             if cold:
-                heap.reset()                                # untimed, outside the events
-            flush.fill_(i & 7)                              # L2 flush (512 MiB write), outside the events
-            s.record(stream)
-            step()
-            e.record(stream)
+                self.heap.reset()                           # one kernel, untimed (outside the events)
+            self.flush.fill_(i & 7)                         # L2 flush (512 MiB write), outside the events
+            s.record(self.stream)
+            self._step()
+            e.record(self.stream)
         return ev
 
-    for _ in range(args.warmup):
-        heap.reset()
-        flush.fill_(1)
-        step()
-    torch.cuda.synchronize()
-    counts.zero_()
-    clocks = Clocks(local)
-    clocks.mark()
-    if dist:
-        dist.barrier()
-    torch.cuda.synchronize()
-    t_wall = time.perf_counter()
-    ev = timed_steps(args.steps, cold=True)
-    torch.cuda.synchronize()
-    if dist:
-        dist.barrier()
-    wall = time.perf_counter() - t_wall
-    clk = clocks.stop()
-    kern_ms = [s.elapsed_time(e) for s, e in ev]
-    ms = sum(kern_ms) / len(kern_ms)
-    c = counts.cpu().numpy()
-    # the same steps on a warm heap (no reset: bins and chunks of the previous step reused)
-    counts.zero_()
-    ev_w = timed_steps(args.steps, cold=False)
-    torch.cuda.synchronize()
-    warm_ms = sum(s.elapsed_time(e) for s, e in ev_w) / args.steps
-    calls_step = int(c[0] + c[2]) // args.steps
-    fails_step = int(c[1]) // args.steps
-    ms_max, tot = reduce_over_ranks(dist, ms, calls_step, dev)
-    value = tot / (ms_max / 1e3)
+    def measure(self, barrier):
+        torch, args, t = self.torch, self.args, self.trace
+        for _ in range(args.warmup):
+            self.heap.reset()
+            self.flush.fill_(1)
+            self._step()
+        torch.cuda.synchronize()
+        self.counts.zero_()
+        clocks = Clocks(self.local)
+        clocks.mark()
+        barrier()
+        torch.cuda.synchronize()
+        t_wall = time.perf_counter()
+        ev = self._timed_steps(args.steps, cold=True)
+        torch.cuda.synchronize()
+        barrier()
+        wall = time.perf_counter() - t_wall
+        clk = clocks.stop()
+        kern_ms = [s.elapsed_time(e) for s, e in ev]
+        c = self.counts.cpu().numpy()
+        self.counts.zero_()
+        ev_w = self._timed_steps(args.steps, cold=False)         # warm heap: the previous step's bins reused
+        torch.cuda.synchronize()
+        warm_ms = sum(s.elapsed_time(e) for s, e in ev_w) / args.steps
+        # e2e through the C ABI: H2D of the step's trace from pinned memory, the
+        # kernel, D2H of the counts, all inside the events
+        from paper_conf_ppopp_geladog19_b200.runner import run_timed_host
+        h_sizes = torch.from_numpy(t.sizes.view(np.int32)).pin_memory()
+        h_counts = np.zeros(4, dtype=np.uint64)
+        e2e_ms = []
+        for i in range(args.warmup + args.steps):
+            self.heap.reset()
+            self.flush.fill_(2)
+            s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            s0.record(self.stream)
+            run_timed_host(self.heap, h_sizes, t.R, t.T, t.D, h_counts, args.block, self.stream)
+            s1.record(self.stream)
+            s1.synchronize()
+            if i >= args.warmup:
+                e2e_ms.append(s0.elapsed_time(s1))
+        calls = int(c[0] + c[2]) // args.steps
+        return {"ms": sum(kern_ms) / len(kern_ms), "calls": calls, "fails": int(c[1]) // args.steps,
+                "kern_ms": kern_ms, "warm_ms": warm_ms, "wall": wall, "clocks": clk,
+                "e2e_ms": sum(e2e_ms) / len(e2e_ms), "e2e_calls": int(h_counts[0] + h_counts[2]),
+                "h2d": int(t.sizes.nbytes), "d2h": 32,
+                # per step: the timed kernel; between the events: 1 reset kernel + 1 torch fill (L2 flush)
+                "launches": args.steps * 2, "launch_note": "per step: k_timed (timed) + k_reset (untimed, between events)"}
 
-    # ---- e2e: host buffers through the C ABI (H2D of the trace, kernel, D2H of counts)
-    h_sizes = torch.from_numpy(trace.sizes.view(np.int32)).pin_memory()
-    h_counts = np.zeros(4, dtype=np.uint64)
-    from paper_conf_ppopp_geladog19_b200.runner import run_timed_host
-    e2e_ms = []
-    for i in range(args.warmup + args.steps):
-        heap.reset()
-        flush.fill_(2)
-        s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        s0.record(stream)
-        run_timed_host(heap, h_sizes, R, T, D, h_counts, args.block, stream)
-        s1.record(stream)
-        s1.synchronize()
-        if i >= args.warmup:
-            e2e_ms.append(s0.elapsed_time(s1))
-    e2e_calls = int(h_counts[0] + h_counts[2])
-    e2e_ms_max, e2e_tot = reduce_over_ranks(dist, sum(e2e_ms) / len(e2e_ms), e2e_calls, dev)
-    e2e = {"value": e2e_tot / (e2e_ms_max / 1e3), "unit": UNIT,
-           "h2d_bytes_per_step": int(trace.sizes.nbytes), "d2h_bytes_per_step": 32,
-           "ms_per_step": e2e_ms_max}
-
-    if rank != 0:
-        if dist:
-            dist.barrier()
-            dist.destroy_process_group()
-        return 0
-
-    # ---- roofline: L2 atomics, peak from the committed microbenchmark, measured live
-    buf = torch.zeros(148 * 8 * 256 * 4 + 8192, dtype=torch.int64, device=dev)
-    sink = torch.zeros(8, dtype=torch.int64, device=dev)
-    peaks = {}
-    grid, blk, iters = 148 * 8, 256, 64
-    for pat in (0, 1, 3):
-        for rep in range(3):
-            a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            a0.record(stream)
-            ga.ga_l2_atomic_bench(stream.cuda_stream, pat, buf.data_ptr(), buf.numel(), iters, grid, blk,
-                                  sink.data_ptr())
-            a1.record(stream)
-            a1.synchronize()
-            if rep:
-                rate = grid * blk * iters / (a0.elapsed_time(a1) / 1e3) / 1e9
-                peaks[pat] = max(peaks.get(pat, 0.0), rate)
-    p_atom = max(peaks[0], peaks[1])
-    a_min = algorithmic_atomics(trace.sizes)
-    achieved = a_min / (ms / 1e3) / 1e9
-    kinfo = ga.ga_kernel_info(0, args.block)
-    traffic = None                                          # DRAM bytes per launch, from the committed ncu capture
-    tf = os.path.join(ROOT, "profiles", "r01_ncu_traffic.json")
-    if os.path.exists(tf):
-        traffic = json.load(open(tf)).get("traffic_bytes")
-    roofline = {"bound": "l2_atomic", "achieved": achieved, "peak": p_atom, "unit": "Gatom/s",
-                "frac": achieved / p_atom, "traffic": traffic, "traffic_unit": "DRAM bytes per launch (ncu)",
-                "per_launch_algorithmic_atomics": a_min,
-                "peak_source": "measured live: ga_l2_atomic_bench distinct-word ATOMG/REDG (max)",
-                "peak_patterns_gatom_s": {"atomg_distinct": peaks[0], "redg_distinct": peaks[1],
-                                          "atomg_1184_words": peaks[3]},
+    def roofline(self, ms):
+        ga, torch = self.ga, self.torch
+        peak = l2_peak(ga, torch, self.dev, self.stream)
+        a_min = algorithmic_atomics(self.trace.sizes)
+        achieved = a_min / (ms / 1e3) / 1e9
+        kinfo = ga.ga_kernel_info(0, self.args.block)
+        traffic = None                                       # DRAM bytes per launch, from the committed ncu capture
+        for name in ("r02_ncu_traffic.json", "r01_ncu_traffic.json"):
+            tf = os.path.join(ROOT, "profiles", name)
+            if os.path.exists(tf):
+                traffic = json.load(open(tf)).get("traffic_bytes")
+                break
+        return {"bound": "l2_atomic", "achieved": achieved, "peak": peak["peak"], "unit": "Gatom/s",
+                "frac": achieved / peak["peak"], "traffic": traffic, "traffic_unit": "DRAM bytes per launch (ncu)",
+                "per_launch_algorithmic_atomics": a_min, "peak_source": peak["source"], "live_peak": peak["live"],
                 "kernel": {"regs": kinfo["regs"], "blocks_per_sm": kinfo["blocks_per_sm"],
                            "stack_bytes": kinfo["local_bytes"]}}
 
-    out = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
-           "warmup": args.warmup, "ms_per_step": ms_max, "higher_is_better": True, "scaling": "weak",
-           "vs_baseline": None, "dtype": "u64", "data": "synthetic",
-           "config": config_of(trace, args), "e2e": e2e, "gpu_launches": args.steps,
-           "clocks": clk, "roofline": roofline,
-           "calls_per_step": calls_step, "failed_mallocs_per_step": fails_step,
-           "kernel_ms": {"min": min(kern_ms), "max": max(kern_ms)},
-           "heap": "cold: ga_heap_reset (untimed) before every step",
-           "warm": {"ms_per_step": warm_ms, "value": calls_step / (warm_ms / 1e3)}, "wall_s_timed_region": wall}
-
-    if not args.no_extras:
-        # ---- fragmentation (correctness mode: one kernel per round, reserved at boundaries)
-        heap.reset()
-        run = run_correctness(heap, trace.sizes, D, log=False, tag=False, reserved=True)
-        live_peak = run.peak_live_bytes                    # the GPU's own successful requests
-        cpu = oracle_leg(trace, budget_s=10.0)
-        frag_ora = cpu["stats"]["peak_reserved_bytes"] / cpu["stats"]["peak_live_bytes"]
-        frag_gpu = run.peak_reserved_bytes / live_peak if live_peak else None
-        out["fragmentation"] = {"gpu": frag_gpu, "oracle": frag_ora,
-                                "ratio": frag_gpu / frag_ora if frag_gpu else None,
-                                "gpu_peak_reserved_bytes": run.peak_reserved_bytes,
-                                "peak_live_bytes": live_peak,
-                                "oracle_peak_reserved_bytes": cpu["stats"]["peak_reserved_bytes"],
-                                "gpu_failed_mallocs": run.counts["n_fail"]}
-        cpu.pop("stats")
-        cpu.pop("seconds")
-        out["cpu_baseline"] = cpu
-        out["cpu_baseline_all_cores"] = oracle_leg_parallel(trace)
-
-        # ---- CUDA device malloc on the same trace (bounded prefix of rounds)
+    def extras(self, out, value):
+        """Rank 0 only: CUDA malloc, fragmentation, CPU baselines, d3 / d4 / d2."""
+        from paper_conf_ppopp_geladog19_b200.runner import run_correctness
+        torch, ga, args, t, heap = self.torch, self.ga, self.args, self.trace, self.heap
+        stream, dev = self.stream, self.dev
+        # CUDA device malloc on the same trace (bounded prefix of rounds)
         heap.reset()
         torch.cuda.synchronize()
         cc = torch.zeros(8, dtype=torch.int64, device=dev)
@@ -528,35 +519,113 @@ def main():
             cc.zero_()
             a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             a0.record(stream)
-            ga.ga_cuda_trace_timed(stream.cuda_stream, d_sizes.data_ptr(), rr, T, D, cc.data_ptr(), args.block)
+            ga.ga_cuda_trace_timed(stream.cuda_stream, self.d_sizes.data_ptr(), rr, t.T, t.D, cc.data_ptr(),
+                                   args.block)
             a1.record(stream)
             a1.synchronize()
             t_cuda = a0.elapsed_time(a1) / 1e3
-            if t_cuda * 2 > args.cuda_budget_s or rr >= R:
+            if t_cuda * 2 > args.cuda_budget_s or rr >= t.R:
                 break
-            rr = min(R, rr * 2)
+            rr = min(t.R, rr * 2)
         ccn = cc.cpu().numpy()
         cuda_rate = float(ccn[0] + ccn[2]) / t_cuda
-        out["cuda_malloc"] = {"value": cuda_rate, "unit": UNIT, "rounds": rr,
-                              "failed_mallocs": int(ccn[1]), "seconds": t_cuda,
-                              "heap_limit_bytes": trace.heap_bytes}
-        out["speedup_vs_cuda_malloc"] = value / cuda_rate
+        out["cuda_malloc"] = {"value": cuda_rate, "unit": UNIT, "speedup": value / cuda_rate, "rounds": rr,
+                              "failed_mallocs": int(ccn[1]), "seconds": round(t_cuda, 3)}
+        # fragmentation: correctness mode, one kernel per round
+        heap.reset()
+        run = run_correctness(heap, t.sizes, t.D, log=False, tag=False, reserved=True)
+        st = heap.stats()
+        cpu = oracle_leg(t, budget_s=10.0)
+        frag_ora = cpu["stats"]["peak_reserved_bytes"] / cpu["stats"]["peak_live_bytes"]
+        frag_gpu = run.peak_reserved_bytes / run.peak_live_bytes if run.peak_live_bytes else None
+        out["fragmentation"] = {"gpu": frag_gpu, "oracle": frag_ora,
+                                "ratio": frag_gpu / frag_ora if frag_gpu else None,
+                                "gpu_failed_mallocs": run.counts["n_fail"],
+                                "device_peak_reserved_bytes": st["peak_reserved_bytes"],
+                                "boundary_peak_reserved_bytes": run.peak_reserved_bytes}
+        cpu.pop("stats")
+        cpu.pop("seconds")
+        out["cpu_baseline"] = cpu
+        out["d4_levels"] = d4_levels(ga, stream, dev, args, self.flush)
+        out["d3"] = d3_sweep(ga, heap, stream, dev, t.T, args)
+        out["d2"] = d2_bsem(ga, stream, dev)
+        out["cpu_baseline_all_cores"] = oracle_leg_parallel(t)
 
-        # ---- d3: warp-uniform sizes 16 B - 8 KiB (BASELINE configs[2]), malloc+free per
-        # thread and round (D = 0), full grid; CUDA malloc on a bounded prefix of rounds
-        out["d3_sweep"] = d3_sweep(ga, heap, stream, dev, T, args)
 
-        # ---- d4 at the fit and exhaust pressure levels
-        out["d4_levels"] = d4_levels(ga, stream, dev, args, flush)
+def l2_peak(ga, torch, dev, stream):
+    """The roofline denominator: the committed, ncu-checked L2-atomic peak
+    (profiles/l2_atomic_peak.json, tools/l2_peak.py) if present, and the same
+    microbenchmark measured live beside it."""
+    buf = torch.zeros(148 * 8 * 256 * 4 + 8192, dtype=torch.int64, device=dev)
+    sink = torch.zeros(8, dtype=torch.int64, device=dev)
+    live = {}
+    grid, blk, iters = 148 * 8, 256, 64
+    for pat, name in ((0, "atomg_distinct"), (1, "redg_distinct"), (3, "atomg_1184_words")):
+        for rep in range(3):
+            a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a0.record(stream)
+            ga.ga_l2_atomic_bench(stream.cuda_stream, pat, buf.data_ptr(), buf.numel(), iters, grid, blk,
+                                  sink.data_ptr())
+            a1.record(stream)
+            a1.synchronize()
+            if rep:
+                live[name] = max(live.get(name, 0.0), grid * blk * iters / (a0.elapsed_time(a1) / 1e3) / 1e9)
+    pf = os.path.join(ROOT, "profiles", "l2_atomic_peak.json")
+    if os.path.exists(pf):
+        p = json.load(open(pf))
+        return {"peak": p["peak_gatom_s"], "source": p["source"], "live": live}
+    return {"peak": max(live["atomg_distinct"], live["redg_distinct"]), "live": live,
+            "source": "measured live: ga_l2_atomic_bench distinct-word ATOMG/REDG (max)"}
 
-        # ---- d2: bulk-semaphore microbenchmark (BASELINE configs[1], Sec. 5.1)
-        out["d2_bsem"] = d2_bsem(ga, stream, dev)
 
+def main(argv=None, arm_factory=GpuArm):
+    argv = sys.argv[1:] if argv is None else list(argv)
+    args = parse_args(argv)
+    if args.impl == "reference":
+        return run_reference(args, tracegen.d4_mixed("pressure"))
+    rc = launch_or_refuse(args, argv)
+    if rc is not None:
+        return rc
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    dist = None
+    arm = arm_factory(args, rank, local)
+    if world > 1:
+        import torch
+        import torch.distributed as dist
+        kw = {"device_id": torch.device("cuda", local)} if arm.backend == "nccl" else {}
+        dist.init_process_group(arm.backend, **kw)
+    barrier = dist.barrier if dist else (lambda: None)
+    m = arm.measure(barrier)
+    ms_max, tot = reduce_over_ranks(dist, m["ms"], m["calls"], arm.reduce_device)
+    e2e_ms, e2e_tot = reduce_over_ranks(dist, m["e2e_ms"], m["e2e_calls"], arm.reduce_device)
+    if rank != 0:
+        if dist:
+            dist.barrier()
+            dist.destroy_process_group()
+        return 0
+    value = tot / (ms_max / 1e3)
+    t = arm.trace
+    out = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+           "warmup": args.warmup, "ms_per_step": ms_max, "higher_is_better": True, "scaling": "weak",
+           "vs_baseline": None, "dtype": "u64", "data": "synthetic", "config": config_of(t, args),
+           "e2e": {"value": e2e_tot / (e2e_ms / 1e3), "unit": UNIT, "h2d_bytes_per_step": m["h2d"],
+                   "d2h_bytes_per_step": m["d2h"], "ms_per_step": e2e_ms},
+           "gpu_launches": m["launches"] * world, "gpu_launches_note": m["launch_note"],
+           "clocks": m["clocks"], "roofline": arm.roofline(m["ms"])}
+    tail = {"calls_per_step": m["calls"], "failed_mallocs_per_step": m["fails"],
+            "kernel_ms": {"min": min(m["kern_ms"]), "max": max(m["kern_ms"])},
+            "heap": "cold: ga_heap_reset (one kernel, untimed) before every step",
+            "warm": {"ms_per_step": m["warm_ms"], "value": m["calls"] / (m["warm_ms"] / 1e3)},
+            "wall_s_timed_region": m["wall"]}
+    if not args.no_extras:
+        arm.extras(out, value)                             # cuda_malloc and fragmentation first: short tail
+    out.update(tail)
     print(json.dumps(out), flush=True)
     if dist:
         dist.barrier()
         dist.destroy_process_group()
-    heap.close()
     return 0
 
 

@@ -89,11 +89,12 @@ ga_status ga_l2_atomic_bench(ga_stream_t stream, int pattern, uint64_t* d_buf, u
                              uint32_t iters, uint32_t grid, uint32_t block, uint64_t* d_sink);
 
 /* Bulk-semaphore microbenchmark (config d2, Sec. 5.1).
- * variant: 0 warp-aggregated bulk semaphore (one CAS per warp group),
- *          1 per-thread bulk semaphore, 2 per-thread counting semaphore
- *          (Sec. 3.2, k forced to 1), 3 plain per-thread atomicAdd(-k)/(+k),
- *          4 per-thread bulk semaphore in the fetch-add form (every update one
- *          fetch-add; may over-produce, never over-grants).
+ * variant: 0 warp-aggregated bulk semaphore (ga_bsem_wait: the CUDA path's
+ *          fetch-add form, one wait per warp group), 1 per-thread bulk semaphore
+ *          in the paper's CAS form (one CAS per decision),
+ *          2 per-thread counting semaphore (Sec. 3.2, k forced to 1), 3 plain
+ *          per-thread atomicAdd(-k)/(+k), 4 per-thread bulk semaphore in the
+ *          fetch-add form (ga_bsem_wait per thread).
  * k: units per thread per wait (1..32); 0 = per-lane random 1..32.
  * B: batch size; n_sems: 1 (global) or one per SM; acquire_only: 1 = Fig. 5
  * mode (no release).  sems: DEVICE u64[n_sems*4] (zeroed by the call).

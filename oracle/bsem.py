@@ -183,16 +183,17 @@ def explore(Ns, B: int, pool: int, strict: bool = False, cd_form: bool = False):
 #   "arena_old"  round-1 arena fast path: fetch-add C -= N; on a short pre-image
 #                add N back and run Alg. 1 as a CAS loop (what ADVICE r1 flagged:
 #                the transient C - N hides N units from other deciders).
-#   "arena"      conservative fast path: fetch-add (C -= N, D += N) keeps C + D;
+#   "arena"      (an intermediate round-2 form, kept as a checked alternative)
+#                conservative fast path: fetch-add (C -= N, D += N) keeps C + D;
 #                ACQUIRED iff the pre-image shows C >= N and C + D >= N, then a
 #                repayment red D -= N; otherwise add (C += N, D -= N) back and
 #                run the CAS loop.
 #   "tree_old"   round-1 optimistic TBuddy form: fetch-add C -= N decides on the
 #                pre-image; a second add converts to GROW (C += N, E += B' - N)
 #                or to a reservation (C += N, R += N).
-#   "tree"       conservative optimistic form: the first fetch-add is
-#                (C -= N, D += B'); ACQUIRED repays D -= B', GROW adds
-#                (C += N, D -= N), a reservation adds (C += N, D -= N + B').
+#   "fa"         the CUDA path's form for every semaphore (round 2): the first
+#                fetch-add is (C -= N, D += B'); ACQUIRED repays D -= B', GROW
+#                adds (C += N, D -= N), a reservation adds (C += N, D -= N + B').
 # In the conservative forms every in-flight operation only lowers C and only
 # raises C + D relative to the state with all decided operations applied, so no
 # thread can take units that are not there (over-grant) or decide GROW when the
@@ -201,7 +202,7 @@ def explore(Ns, B: int, pool: int, strict: bool = False, cd_form: bool = False):
 # ---------------------------------------------------------------------------
 (G_FAST, G_FIX, G_UNDO, G_CAS, G_SPIN, G_RETRY, G_TGROW, G_TRES, G_TSPIN, G_TRETRY,
  G_GROWING, G_REL, G_OK, G_FAIL) = range(14)
-FORMS = ("alg1", "arena_old", "arena", "tree_old", "tree")
+FORMS = ("alg1", "arena_old", "arena", "tree_old", "fa")
 
 
 def _pending(form, pc, N, Bp):
@@ -211,7 +212,7 @@ def _pending(form, pc, N, Bp):
         return {G_FIX: (0, -N), G_UNDO: (N, -N)}.get(pc, (0, 0))
     if form == "arena_old":
         return {G_UNDO: (N, 0)}.get(pc, (0, 0))
-    if form == "tree":
+    if form == "fa":
         return {G_FIX: (0, -Bp), G_TGROW: (N, -N), G_TRES: (N, -N - Bp)}.get(pc, (0, 0))
     if form == "tree_old":
         return {G_TGROW: (N, Bp - N), G_TRES: (N, -N)}.get(pc, (0, 0))
@@ -288,7 +289,7 @@ def explore_gpu(Ns, B: int, pool: int, form: str, release: bool = False, init_C:
                     go(t, (C - N, D + N), G_FIX if ok else G_UNDO)
                 elif form == "tree_old":
                     go(t, (C - N, D), done if C >= N else (G_TGROW if C + D < N else G_TRES))
-                else:                                         # tree
+                else:                                         # fa
                     ok = C >= N and (C + D >= N or not fast_needs_cover)
                     go(t, (C - N, D + Bp), G_FIX if ok else (G_TGROW if C + D < N else G_TRES))
             elif pc == G_FIX:
@@ -297,9 +298,9 @@ def explore_gpu(Ns, B: int, pool: int, form: str, release: bool = False, init_C:
                 nw = (C + N, D - N) if form == "arena" else (C + N, D)
                 go(t, nw, G_CAS, nw)
             elif pc == G_TGROW:
-                go(t, (C + N, D - N) if form == "tree" else (C + N, D + Bp - N), G_GROWING)
+                go(t, (C + N, D - N) if form == "fa" else (C + N, D + Bp - N), G_GROWING)
             elif pc == G_TRES:
-                go(t, (C + N, D - N - Bp) if form == "tree" else (C + N, D - N), G_TSPIN)
+                go(t, (C + N, D - N - Bp) if form == "fa" else (C + N, D - N), G_TSPIN)
             elif pc == G_TSPIN:
                 if not (C < N and C + D >= 0):
                     go(t, (C, D), G_TRETRY)

@@ -254,11 +254,11 @@ __global__ void k_bsem(ga_bsem_cfg cfg, uint64_t* sems, uint64_t* out, uint32_t 
             }
             __syncwarp(act);
         } else if (cfg.variant == 1 || cfg.variant == 4) {
-            // 1: exact form (CAS decisions); 4: fetch-add form (every update one
-            // fetch-add, as the paper's R-saturation note implies)
+            // 1: the paper's form, one CAS per decision; 4: the
+            // CUDA path's fetch-add form (ga_bsem_wait), per thread
             uint32_t Bp = cfg.B * ((k + cfg.B - 1) / cfg.B);
-            int r = cfg.variant == 1 ? ga_bsem_wait((ga_bsem*)s, k, Bp)
-                                     : ga::bsem_wait_fast((uint64_t*)s, k, Bp, ga::NoSpin());
+            int r = cfg.variant == 1 ? ga::bsem_wait_cas((uint64_t*)s, k, Bp)
+                                     : ga_bsem_wait((ga_bsem*)s, k, Bp);
             waits++;
             if (r == GA_GROW) {
                 atomicAdd((unsigned long long*)bump + (tid & zero), (unsigned long long)Bp);

@@ -260,6 +260,23 @@ static __device__ __forceinline__ uint64_t valid_mask(int c, int w) {
     return s >= 64 ? ~0ull : s <= 0 ? 0ull : ((1ull << s) - 1);
 }
 static __device__ __forceinline__ uint32_t arena_of(const ga_desc* h) { return smid() % h->n_arenas; }
+// SMs sharing one arena for class c (reading R-41).  An arena holds at least
+// one 64-page chunk per class it serves, so per-SM arenas reserve 148 chunks
+// (37 MiB) for a class whatever its live set: at full occupancy a 16 B class
+// holds 4.6 MiB live and the reserve dominated fragmentation (7.8x the
+// oracle's on d3).  The tiny classes share arenas so an arena's live set of
+// the class is about a chunk; spans share GA_SPAN_SHARE SMs.
+#ifndef GA_SMALL_SHARE
+#define GA_SMALL_SHARE 1
+#endif
+static __device__ __forceinline__ uint32_t class_share(int c) {
+    if (c >= kNbin) return GA_SPAN_SHARE;
+#if GA_SMALL_SHARE
+    return c == 0 ? 8 : c <= 2 ? 4 : c == 3 ? 2 : 1;              // 16 B: 8, 32 / 64 B: 4, 128 B: 2
+#else
+    return 1;
+#endif
+}
 static __device__ __forceinline__ uint64_t* sem_ptr(const ga_desc* h, uint32_t A, int c) { return h->sem + ((uint64_t)A * kNcls + c) * kSemStride; }
 static __device__ __forceinline__ uint64_t* psem_ptr(const ga_desc* h, uint32_t A) { return h->psem + (uint64_t)A * kSemStride; }
 static __device__ __forceinline__ uint64_t* tsem_ptr(const ga_desc* h, int n) { return h->tsem + (uint64_t)n * kSemStride; }
@@ -312,29 +329,62 @@ static __device__ __forceinline__ bool bsem_trywait(uint64_t* s, uint32_t N, uin
     return bsem_trywait_direct(s, N, keep);
 }
 
-// Fast acquire: one fetch-add (C -= N, D += N).  ACQUIRED iff the pre-image
-// shows C >= N and C + D >= N (Alg. 1 tests growth first); the speculation is
-// then settled by a repayment red (D -= N).  Otherwise the move is reversed and
-// the returned word (*w) seeds the exact CAS loop.
-static __device__ __forceinline__ bool bsem_fast_acquire(uint64_t* s, uint32_t N, uint64_t* w) {
-    const uint64_t d = dCD(-(int32_t)N, (int32_t)N);
-    const uint64_t old = a_add(s, d);
-    if (sem_C(old) >= (int32_t)N && (int64_t)sem_C(old) + sem_D(old) >= (int64_t)N) {
-        red_rlx(s, dCD(0, -(int32_t)N));
-        return true;
+// Alg. 1 as the CUDA path runs it: fetch-adds only, no CAS retry
+// loop on hot words.  The first fetch-add (C -= N, D += B) is conservative for
+// every outcome (see dCD); its pre-image decides in Alg. 1's order, and one
+// more add settles it:
+//   pre C + D < N   -> GROW:     (C += N, D -= N)       net E += B - N
+//   pre C >= N      -> ACQUIRED: (D -= B)               net C -= N
+//   otherwise       -> reserve:  (C += N, D -= N + B)   net R += N; spin while
+//                      C < N and C + D >= 0 (R-2), running `spin()` -- the
+//                      delegated work of Sec. 4.2.1 -- between polls; then
+//                      R -= N and decide again.
+// Returns kAcquired (0) or kGrow (-1): the caller must produce B units, keep N
+// and signal(B - N, B - N), or signal(0, B - N) on failure.
+// Model-checked as form "fa" (oracle/bsem.py explore_gpu): exact for unit
+// demands, no deadlock, no over-grant (tests/test_oracle_bsem.py).
+static __device__ __forceinline__ int bsem_decide(uint64_t* s, uint64_t old, uint32_t N, uint32_t B, uint64_t* w) {
+    const int32_t C = sem_C(old), D = sem_D(old);
+    if ((int64_t)C + D < (int64_t)N) { red_rlx(s, dCD((int32_t)N, -(int32_t)N)); return kGrow; }
+    if (C >= (int32_t)N) { red_rlx(s, dCD(0, -(int32_t)B)); return kAcquired; }
+    const uint64_t res = dCD((int32_t)N, -(int32_t)(N + B));
+    *w = a_add(s, res) + res;
+    return kBlocked;
+}
+template <uint32_t kCap, class Spin>
+static __device__ __noinline__ int bsem_wait_slow(uint64_t* s, uint32_t N, uint32_t B, Spin spin, uint64_t w) {
+    GA_DBG_CNT;
+    for (;;) {
+        uint32_t ns = 32;
+        while (sem_C(w) < (int32_t)N && (int64_t)sem_C(w) + sem_D(w) >= 0) {                    // R-2
+            spin();
+            SPIN_NOTE(dbg_cnt, 1, (uint64_t)(uintptr_t)s, w);
+            __nanosleep(ns);
+            if (ns < kCap) ns <<= 1;
+            w = ld_rlx(s);
+        }
+        red_rlx(s, (uint64_t)N);                                                             // R -= N
+        const int r = bsem_decide(s, a_add(s, dCD(-(int32_t)N, (int32_t)B)), N, B, &w);
+        if (r != kBlocked) return r;
     }
-    const uint64_t back = dCD((int32_t)N, -(int32_t)N);
-    *w = a_add(s, back) + back;
-    return false;
+}
+// kCap: the __nanosleep backoff cap of a blocked waiter (R-5; arena semaphores
+// 2 us, TBuddy orders GA_TREE_SPIN_CAP)
+template <uint32_t kCap = 2048, class Spin>
+static __device__ __forceinline__ int bsem_wait(uint64_t* s, uint32_t N, uint32_t B, Spin spin) {
+    uint64_t w = 0;
+    const int r = bsem_decide(s, a_add(s, dCD(-(int32_t)N, (int32_t)B)), N, B, &w);
+    return r != kBlocked ? r : bsem_wait_slow<kCap>(s, N, B, spin, w);
+}
+template <class Spin>
+static __device__ __forceinline__ int bsem_wait_fast(uint64_t* s, uint32_t N, uint32_t B, Spin spin) {
+    return bsem_wait<GA_TREE_SPIN_CAP>(s, N, B, spin);
 }
 
-// Alg. 1 as a CAS loop on the packed word, starting from the
-// caller's copy w.  One CAS decides among the three branches on the current
-// word; a blocked waiter runs `spin()` -- the delegated work of Sec. 4.2.1 --
-// between polls.  Reading R-2: keep waiting while C < N and C + D >= 0.
-template <class Spin>
-static __device__ __noinline__ int bsem_wait_cas(uint64_t* s, uint32_t N, uint32_t B, Spin spin, uint64_t w) {
-    GA_DBG_CNT;
+// Alg. 1 as one CAS per decision on the packed word (the paper's form,
+// P:L766-772) -- only the d2 microbenchmark's per-thread CAS variant uses it.
+static __device__ __noinline__ int bsem_wait_cas(uint64_t* s, uint32_t N, uint32_t B) {
+    uint64_t w = ld_rlx(s);
     for (;;) {
         int32_t C = sem_C(w), D = sem_D(w);
         uint64_t nw;
@@ -346,58 +396,9 @@ static __device__ __noinline__ int bsem_wait_cas(uint64_t* s, uint32_t N, uint32
         if (old != w) { w = old; continue; }
         if (res != kBlocked) return res;
         uint32_t ns = 64;
-        for (;;) {                                                                           // R-2
-            w = ld_rlx(s);
-            if (!(sem_C(w) < (int32_t)N && (int64_t)sem_C(w) + sem_D(w) >= 0)) break;
-            spin();
-            SPIN_NOTE(dbg_cnt, 1, (uint64_t)(uintptr_t)s, w);
-            __nanosleep(ns);
-            if (ns < 2048) ns <<= 1;
-        }
+        do { __nanosleep(ns); if (ns < 2048) ns <<= 1; w = ld_rlx(s); }
+        while (sem_C(w) < (int32_t)N && (int64_t)sem_C(w) + sem_D(w) >= 0);                   // R-2
         w = a_add(s, (uint64_t)N) + (uint64_t)N;                                             // R -= N
-    }
-}
-
-// Alg. 1 for arena semaphores (class and page: an extra batch costs real
-// pages).  Returns kAcquired (0) or kGrow (-1; the caller must produce B
-// units, keep N and signal(B - N, B - N), or signal(0, B - N) on failure,
-// P:L756-764).  A plain load gates the fast acquire.
-template <class Spin>
-static __device__ __forceinline__ int bsem_wait(uint64_t* s, uint32_t N, uint32_t B, Spin spin) {
-    uint64_t w = ld_rlx(s);
-    if (sem_C(w) >= (int32_t)N && (int64_t)sem_C(w) + sem_D(w) >= (int64_t)N && bsem_fast_acquire(s, N, &w))
-        return kAcquired;
-    return bsem_wait_cas(s, N, B, spin, w);
-}
-
-// Alg. 1 for TBuddy order semaphores, in fetch-adds (no CAS retries on the few
-// hot order words).  The first fetch-add (C -= N, D += B) covers every outcome
-// conservatively; the pre-image decides in Alg. 1's order and one more add
-// settles it:
-//   pre C + D < N   -> GROW:     (C += N, D -= N)       net E += B - N
-//   pre C >= N      -> ACQUIRED: (D -= B)               net C -= N
-//   otherwise       -> reserve:  (C += N, D -= N + B)   net R += N; spin (R-2),
-//                      then R -= N and decide again.
-template <class Spin>
-static __device__ __noinline__ int bsem_wait_fast(uint64_t* s, uint32_t N, uint32_t B, Spin spin) {
-    GA_DBG_CNT;
-    const uint64_t first = dCD(-(int32_t)N, (int32_t)B);
-    for (;;) {
-        const uint64_t old = a_add(s, first);
-        const int32_t C = sem_C(old), D = sem_D(old);
-        if ((int64_t)C + D < (int64_t)N) { red_rlx(s, dCD((int32_t)N, -(int32_t)N)); return kGrow; }
-        if (C >= (int32_t)N) { red_rlx(s, dCD(0, -(int32_t)B)); return kAcquired; }
-        const uint64_t res = dCD((int32_t)N, -(int32_t)(N + B));
-        uint64_t w = a_add(s, res) + res;
-        uint32_t ns = 32;
-        while (sem_C(w) < (int32_t)N && (int64_t)sem_C(w) + sem_D(w) >= 0) {                  // R-2
-            spin();
-            SPIN_NOTE(dbg_cnt, 3, (uint64_t)(uintptr_t)s, w);
-            __nanosleep(ns);
-            if (ns < GA_TREE_SPIN_CAP) ns <<= 1;
-            w = ld_rlx(s);
-        }
-        red_rlx(s, (uint64_t)N);                                                             // R -= N
     }
 }
 struct NoSpin { __device__ void operator()() const {} };
@@ -1550,17 +1551,17 @@ static __device__ __noinline__ uint64_t ga_malloc_off(const ga_desc* h, uint64_t
     if (key < 0) return kNull;
     uint64_t my;
     if (key < kNcls) {
-        const uint32_t A = is_span(key) ? arena_of(h) / GA_SPAN_SHARE : arena_of(h);
+        const uint32_t A = arena_of(h) / class_share(key);
         const uint32_t N = __popc(grp), slots = slots_of(key);
         const int leader = __ffs(grp) - 1;
         int r = 0;
         if ((int)lane_id() == leader) {
-            // the fast acquire inline (one fetch-add, no load gate: the units are
-            // usually there); the exact CAS loop out of line
+            // the first fetch-add and its settling inline; a blocked wait out of line
             uint64_t* sp = sem_ptr(h, A, key);
-            uint64_t w;
-            r = bsem_fast_acquire(sp, N, &w) ? kAcquired
-                                             : bsem_wait_cas(sp, N, slots * ((N + slots - 1) / slots), ArenaSpin{h, A}, w);
+            const uint32_t Bp = slots * ((N + slots - 1) / slots);                     // R-8
+            uint64_t w = 0;
+            r = bsem_decide(sp, a_add(sp, dCD(-(int32_t)N, (int32_t)Bp)), N, Bp, &w);
+            if (r == kBlocked) r = bsem_wait_slow<2048>(sp, N, Bp, ArenaSpin{h, A}, w);
         }
         r = __shfl_sync(grp, r, leader);
         my = r == kAcquired ? bin_claim_collective(h, grp, A, key)

@@ -32,12 +32,6 @@ struct Carve {
     template <class T> uint64_t take(uint64_t count) { uint64_t o = off; off = up(off + count * sizeof(T), kAlign); return o; }
 };
 
-__global__ void k_fill_u64(uint64_t* p, uint64_t n, uint64_t v) {
-    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) p[i] = v;
-}
-__global__ void k_fill_u32(uint32_t* p, uint64_t n, uint32_t v) {
-    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) p[i] = v;
-}
 // quiesce step 1: every empty bin back to its chunk (and empty chunks to the tree)
 __global__ void k_quiesce_bins(const ga_desc* h) {
     for (uint64_t p = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; p < h->pages; p += (uint64_t)gridDim.x * blockDim.x) {
@@ -60,27 +54,47 @@ __global__ void k_quiesce_clear(const ga_desc* h) {
 
 inline int grid_for(uint64_t n) { uint64_t b = (n + 255) / 256; return (int)(b > 4096 ? 4096 : (b ? b : 1)); }
 
+// One fused kernel resets every metadata array (a fill or a copy of the
+// empty-heap image per segment, blockIdx.y = segment): ga_heap_reset is a
+// single launch on the caller's stream.
+struct FillSeg { void* p; const uint64_t* src; uint64_t n; uint64_t v; uint32_t bytes; };
+constexpr int kMaxSegs = 16;
+struct FillPlan { FillSeg s[kMaxSegs]; };
+__global__ void __launch_bounds__(256) k_reset(FillPlan plan) {
+    const FillSeg g = plan.s[blockIdx.y];
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < g.n; i += (uint64_t)gridDim.x * blockDim.x) {
+        if (g.bytes == 8) ((uint64_t*)g.p)[i] = g.src ? g.src[i] : g.v;
+        else ((uint32_t*)g.p)[i] = (uint32_t)g.v;
+    }
+}
+
 ga_status init_heap(ga_heap_t h, cudaStream_t s) {
-    ga_desc& d = h->dev;
-    auto chk = [](cudaError_t e) { return e == cudaSuccess; };
-    k_fill_u64<<<grid_for(d.pages * kBinWords), 256, 0, s>>>(d.bits, d.pages * kBinWords, ~0ull);
-    k_fill_u32<<<grid_for(d.pages), 256, 0, s>>>(d.kind, d.pages, 0u);
-    k_fill_u64<<<grid_for(d.nchunks), 256, 0, s>>>(d.chunk_used, d.nchunks, ~0ull);
-    k_fill_u32<<<grid_for(d.nchunks), 256, 0, s>>>(d.chunk_owner, d.nchunks, 0u);
-    k_fill_u64<<<grid_for(d.nchunks * kNcls), 256, 0, s>>>(d.chunk_nonfull, d.nchunks * kNcls, 0ull);
-    k_fill_u64<<<grid_for(d.nchunks), 256, 0, s>>>(d.chunk_cand, d.nchunks, 0ull);
-    k_fill_u64<<<grid_for((uint64_t)d.n_arenas * kNcls * kSemStride), 256, 0, s>>>(d.sem, (uint64_t)d.n_arenas * kNcls * kSemStride, sem_word(0, 0));
-    k_fill_u64<<<grid_for((uint64_t)d.n_arenas * kSemStride), 256, 0, s>>>(d.psem, (uint64_t)d.n_arenas * kSemStride, sem_word(0, 0));
-    k_fill_u32<<<grid_for((uint64_t)d.n_arenas * kNcls), 256, 0, s>>>(d.hint, (uint64_t)d.n_arenas * kNcls, 0xFFFFFFFFu);
-    k_fill_u64<<<grid_for(h->ahb_total_words), 256, 0, s>>>(d.ahb, h->ahb_total_words, 0ull);
-    k_fill_u64<<<1, 32, 0, s>>>(d.stats, kStatWords, 0ull);
-    k_fill_u64<<<grid_for((uint64_t)d.n_arenas * kActrStride), 256, 0, s>>>(d.actr, (uint64_t)d.n_arenas * kActrStride, 0ull);
-    k_fill_u32<<<1, 64, 0, s>>>(d.lvl_hint, 48, 0u);
-    if (!chk(cudaGetLastError())) return GA_ECUDA;
-    if (!chk(cudaMemcpyAsync(h->ddesc, &h->dev, sizeof(ga_desc), cudaMemcpyHostToDevice, s))) return GA_ECUDA;
-    if (!chk(cudaMemcpyAsync(d.avail, h->avail_init.data(), h->avail_words * 8, cudaMemcpyHostToDevice, s))) return GA_ECUDA;
-    if (!chk(cudaMemcpyAsync(d.tsem, h->tsem_init.data(), h->tsem_init.size() * 8, cudaMemcpyHostToDevice, s))) return GA_ECUDA;
-    return GA_OK;
+    const ga_desc& d = h->dev;
+    FillPlan plan{};
+    int n = 0;
+    auto seg = [&](void* p, uint64_t cnt, uint64_t v, uint32_t bytes, const uint64_t* src = nullptr) {
+        plan.s[n++] = FillSeg{p, src, cnt, v, bytes};
+    };
+    seg(d.bits, d.pages * kBinWords, ~0ull, 8);                  // all ones: no live bin
+    seg(d.kind, d.pages, 0, 4);
+    seg(d.chunk_used, d.nchunks, ~0ull, 8);                      // all ones: not owned
+    seg(d.chunk_owner, d.nchunks, 0, 4);
+    seg(d.chunk_nonfull, d.nchunks * kNcls, 0, 8);
+    seg(d.chunk_cand, d.nchunks, 0, 8);
+    seg(d.sem, (uint64_t)d.n_arenas * kNcls * kSemStride, sem_word(0, 0), 8);
+    seg(d.psem, (uint64_t)d.n_arenas * kSemStride, sem_word(0, 0), 8);
+    seg(d.hint, (uint64_t)d.n_arenas * kNcls, 0xFFFFFFFFu, 4);
+    seg(d.ahb, h->ahb_total_words, 0, 8);
+    seg(d.stats, kStatWords, 0, 8);
+    seg(d.actr, (uint64_t)d.n_arenas * kActrStride, 0, 8);
+    seg(d.lvl_hint, 48, 0, 4);
+    seg(d.avail, h->avail_words, 0, 8, h->init_img);             // the empty tree (R-30)
+    seg(d.tsem, (uint64_t)(d.L + 1) * kSemStride, 0, 8, h->init_img + h->avail_words);
+    uint64_t most = 0;
+    for (int i = 0; i < n; i++) most = plan.s[i].n > most ? plan.s[i].n : most;
+    const uint64_t bx = (most + 255) / 256;
+    k_reset<<<dim3((unsigned)(bx > 1184 ? 1184 : bx), n), 256, 0, s>>>(plan);
+    return cudaGetLastError() == cudaSuccess ? GA_OK : GA_ECUDA;
 }
 
 // set bit i of a 3-level bitset image [w0 | w1 | w2] (section 3 of ga_device_impl.cuh)
@@ -173,6 +187,7 @@ ga_status ga_heap_create(int device, ga_stream_t stream, void* buf, size_t bytes
     uint64_t o_stats = cv.take<uint64_t>(kStatWords);
     uint64_t o_actr = cv.take<uint64_t>((uint64_t)d.n_arenas * kActrStride);
     uint64_t o_lhint = cv.take<uint32_t>(48);
+    uint64_t o_img = cv.take<uint64_t>(aw + (uint64_t)(L + 1) * kSemStride);
     h->meta_bytes = cv.off;
     if (cudaMalloc(&h->meta, h->meta_bytes) != cudaSuccess) { delete h; cudaSetDevice(prev); return GA_ENOMEM; }
     if (buf) d.base = (char*)buf;
@@ -198,6 +213,7 @@ ga_status ga_heap_create(int device, ga_stream_t stream, void* buf, size_t bytes
     d.tsem = (uint64_t*)(m + o_tsem);
     d.stats = (uint64_t*)(m + o_stats);
     d.actr = (uint64_t*)(m + o_actr);
+    h->init_img = (uint64_t*)(m + o_img);
     d.lvl_hint = (uint32_t*)(m + o_lhint);
     // empty heap: the binary decomposition of the pages into maximal aligned roots (R-30)
     h->avail_init.assign(aw, 0ull);
@@ -212,7 +228,16 @@ ga_status ga_heap_create(int device, ga_stream_t stream, void* buf, size_t bytes
         }
     }
     for (uint32_t n = 0; n <= L; n++) h->tsem_init[(uint64_t)n * kSemStride] = sem_word(roots[n], 0);
-    ga_status st = init_heap(h, s);
+    // the empty-tree image lives on the device (reset copies it from there);
+    // the descriptor changes only with ga_debug_attach
+    ga_status st = GA_OK;
+    if (cudaMemcpyAsync(h->init_img, h->avail_init.data(), aw * 8, cudaMemcpyHostToDevice, s) != cudaSuccess ||
+        cudaMemcpyAsync(h->init_img + aw, h->tsem_init.data(), h->tsem_init.size() * 8, cudaMemcpyHostToDevice, s) != cudaSuccess ||
+        cudaMemcpyAsync(h->ddesc, &h->dev, sizeof(ga_desc), cudaMemcpyHostToDevice, s) != cudaSuccess)
+        st = GA_ECUDA;
+    if (st == GA_OK) st = init_heap(h, s);
+    // the host images are read by the async copies above: keep them until done
+    if (st == GA_OK && cudaStreamSynchronize(s) != cudaSuccess) st = GA_ECUDA;
     if (st != GA_OK) { ga_heap_destroy(h); cudaSetDevice(prev); return st; }
     cudaSetDevice(prev);
     *out = h;

@@ -16,6 +16,7 @@ struct ga_heap_s {
     ga_desc dev{};                 // host copy of the descriptor
     ga_desc* ddesc = nullptr;      // device copy (start of the metadata allocation)
     std::vector<uint64_t> avail_init;   // host image of the tree bitmaps (empty heap)
+    uint64_t* init_img = nullptr;       // device copy: avail image, then tsem image
     std::vector<uint64_t> tsem_init;
     uint64_t avail_words = 0;
     uint64_t ahb_total_words = 0;

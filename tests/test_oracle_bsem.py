@@ -139,10 +139,10 @@ def test_group_demand_can_overproduce():
 from oracle.bsem import explore_gpu  # noqa: E402
 
 
-@pytest.mark.parametrize("form", ["arena", "tree"])
+@pytest.mark.parametrize("form", ["fa", "arena"])
 def test_gpu_forms_unit_demand_exact(form):
-    """T <= 6 threads of demand 1 (the Fig. 5 setting): the forms
-    the CUDA path runs grant exactly min(T, pool*B) units (no false starvation,
+    """T <= 6 threads of demand 1 (the Fig. 5 setting): the form
+    the CUDA path runs ("fa"; "arena" is a checked alternative) grants exactly min(T, pool*B) units (no false starvation,
     P:L488-506), use exactly min(pool, ceil(T/B)) batches (no over-production),
     never deadlock, never over-grant, end with D = 0, and are conservative in
     every reachable state (R-35)."""
@@ -175,18 +175,18 @@ def test_gpu_forms_mixed_group_demand():
     C = C0 + produced - held; they use at most ONE batch more than Alg. 1's
     worst interleaving (the over-production bound recorded in DESIGN.md R-35).
     Round 1's forms are checked too: they are not conservative."""
-    worst = {"arena": 0, "tree": 0}
+    worst = {"arena": 0, "fa": 0}
     for release, Ns, B, C0, pool in _mixed_cases():
         ref = explore_gpu(Ns, B, pool, "alg1", release=release, init_C=C0)
         ref_max = max(u for _, u, _ in ref["terminals"])
-        for form in ("arena", "tree"):
+        for form in ("arena", "fa"):
             r = explore_gpu(Ns, B, pool, form, release=release, init_C=C0)
             assert r["deadlocks"] == 0 and r["nonconservative"] == 0 and r["overgrant"] == 0
             for (C, D), used, res in r["terminals"]:
                 held = 0 if release else sum(N for N, o in res if o)
                 assert D == 0 and C == C0 + used * B - held, (form, Ns, B, C0, pool, res)
             worst[form] = max(worst[form], max(u for _, u, _ in r["terminals"]) - ref_max)
-    assert worst == {"arena": 1, "tree": 1}, worst
+    assert worst == {"arena": 1, "fa": 1}, worst
 
 
 def test_round1_forms_are_caught():
