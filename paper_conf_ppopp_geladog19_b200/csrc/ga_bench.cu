@@ -237,7 +237,8 @@ __global__ void k_bsem(ga_bsem_cfg cfg, uint64_t* sems, uint64_t* out, uint32_t 
         uint32_t k = cfg.k ? cfg.k : rnd_k(cfg.seed, tid, it);
         if (cfg.variant == 2) k = 1;
         if (cfg.variant == 0) {
-            unsigned act = __activemask();
+            // masks from __match_any_sync only (ga_device_impl.cuh, active_lanes)
+            unsigned act = ga::active_lanes();
             unsigned grp = __match_any_sync(act, si);
             uint32_t N = __reduce_add_sync(grp, k);
             if ((int)(threadIdx.x & 31) == __ffs(grp) - 1) {
@@ -252,7 +253,7 @@ __global__ void k_bsem(ga_bsem_cfg cfg, uint64_t* sems, uint64_t* out, uint32_t 
                 granted += N;
                 if (!cfg.acquire_only) ga_bsem_signal((ga_bsem*)s, N, 0);
             }
-            __syncwarp(act);
+            (void)__shfl_sync(grp, 0, __ffs(grp) - 1);          // the group waits for its leader
         } else if (cfg.variant == 1 || cfg.variant == 4) {
             // 1: the paper's form, one CAS per decision; 4: the
             // CUDA path's fetch-add form (ga_bsem_wait), per thread

@@ -85,6 +85,9 @@ constexpr int kMaxLevels = 48;
 #ifndef GA_CLAIM_LOCALMASK
 #define GA_CLAIM_LOCALMASK 0     // 1: a group retries the other non-full pages of its chunk before searching again
 #endif
+#ifndef GA_PREFETCH
+#define GA_PREFETCH 1            // 1: the malloc leader loads its block's hinted chunk beside the semaphore fetch-add
+#endif
 #ifndef GA_COUNT_ITERS
 #define GA_COUNT_ITERS 0         // diagnostic: count collective-claim calls / iterations in the repair stats
 #endif
@@ -109,22 +112,23 @@ constexpr int kActrStride = 8;                  // u64 words per arena: [0] mall
 static __device__ __forceinline__ uint32_t lane_id() { uint32_t r; asm volatile("mov.u32 %0, %%laneid;" : "=r"(r)); return r; }
 static __device__ __forceinline__ uint32_t lanemask_lt() { uint32_t r; asm volatile("mov.u32 %0, %%lanemask_lt;" : "=r"(r)); return r; }
 static __device__ __forceinline__ uint32_t smid() { uint32_t r; asm volatile("mov.u32 %0, %%smid;" : "=r"(r)); return r; }
-// Warp masks for the *_sync intrinsics, made opaque to the compiler's
-// uniformity analysis.  Lanes that call the allocator from divergent code
-// compute their masks in separate groups (each from its own __activemask()),
-// and the groups can be merged at a later convergence barrier (BSYNC).  A mask
-// the compiler believes warp-uniform (a ballot result) is then read through a
-// uniform register (R2UR) as if every co-active lane held the same value: on
-// sm_100a some merged lanes skipped a __syncwarp as "already converged" while
-// the others waited in its divergent path -- a hang at two different WARPSYNCs
-// (cuda-gdb, tests/test_gpu_edge.py).  Opaque masks make the compiler check
-// uniformity (REDUX.OR + R2UR P) before shfl / vote / match and take the
-// per-lane collective path (WARPSYNC.COLLECTIVE) when they differ.
-// __syncwarp(mask) is lowered through R2UR whatever the mask, so the allocator
-// does not use it: a following match / ballot on the same mask is the
-// execution barrier, and warp_release() is the publication barrier.
-static __device__ __forceinline__ unsigned opaque_mask(unsigned m) { asm volatile("" : "+r"(m)); return m; }
-static __device__ __forceinline__ unsigned active_lanes() { return opaque_mask(__activemask()); }
+// Warp masks for the *_sync intrinsics (R-42).  Lanes that call the
+// allocator from divergent code enter in separate groups, each with its own
+// __activemask(), and the hardware can merge the groups again at a later
+// convergence barrier (BSYNC).  ptxas treats a vote result (__activemask,
+// __ballot_sync) as warp-uniform: it reads such a mask through one uniform
+// register (R2UR) and skips the synchronisation when "every lane of the mask is
+// active" -- with merged groups holding different masks, some lanes then skip
+// a _sync the others wait in (a hang found by cuda-gdb: a group's leader left
+// alone at a shuffle its lanes had passed).  A __match_any_sync result is not
+// assumed uniform: ptxas checks it (REDUX.OR + R2UR P) and takes the per-lane
+// collective path (WARPSYNC.COLLECTIVE) when co-active lanes differ.  So every
+// mask the allocator passes to a _sync intrinsic is a match result or an AND
+// of match results, taken right after __activemask() (no barrier between), and
+// __syncwarp(mask) is not used at all.
+static __device__ __forceinline__ unsigned active_lanes() { return __match_any_sync(__activemask(), 0u); }
+// the lanes of mask m whose predicate equals this lane's (a ballot, as a match)
+static __device__ __forceinline__ unsigned lanes_where(unsigned m, bool pred) { return __match_any_sync(m, (unsigned)pred); }
 // Every lane of `grp` has performed its prior writes at gpu scope (fence) and
 // reached this point (ballot) before any lane of grp continues: a leader's
 // release signal that follows publishes every lane's writes.
@@ -987,6 +991,12 @@ static __device__ __noinline__ void nfc_repair(const ga_desc* h, uint32_t A, int
         }
 }
 
+// Per block: the chunk (as a page index) a claim of class c last used -- the
+// block's warps share one arena, so this is a copy of the (A, c) hint that
+// costs a shared-memory load instead of an L2 round trip.  Only a hint: its
+// owner and non-full word are validated before use.
+static __shared__ uint32_t s_chunk_hint[kNcls];
+
 // A chunk of arena A with non-full class-c bins, and its non-full page mask:
 // the hint's chunk first, then the (A, c) summary.  Spins until one shows up
 // (the caller holds units, so a free slot exists or is being published).
@@ -1002,7 +1012,7 @@ static __device__ GA_CLAIM_FN uint64_t bin_find_chunk(const ga_desc* h, uint32_t
     if (hp < h->pages) {                                      // the hint's chunk, if still A's
         const uint32_t own = ld_rlx32(&h->chunk_owner[hp >> kChunkShift]);
         uint64_t m = ld_rlx(nonfull_word(h, hp >> kChunkShift, c));
-        if (own == A + 1 && m) { *mask_out = m; return hp >> kChunkShift; }
+        if (own == A + 1 && m) { s_chunk_hint[c] = hp; *mask_out = m; return hp >> kChunkShift; }
     }
     HB3 nb = arena_hb(h, A, kAhbNfc + c);
     uint32_t seed = scatter_seed();
@@ -1019,6 +1029,7 @@ static __device__ GA_CLAIM_FN uint64_t bin_find_chunk(const ga_desc* h, uint32_t
                 uint64_t m = ld_rlx(nonfull_word(h, ch, c));
                 if (own == A + 1 && m) {
                     st_rlx32(&h->hint[A * kNcls + c], (uint32_t)(ch * kChunkPages + (__ffsll((long long)m) - 1)));
+                    s_chunk_hint[c] = (uint32_t)(ch * kChunkPages);
                     *mask_out = m;
                     return ch;
                 }
@@ -1293,7 +1304,8 @@ static __device__ __noinline__ uint64_t bin_malloc_lane(const ga_desc* h, uint32
 // Lanes spread over the chunk's non-full pages by their rank (each thread walks
 // the number of elements its index dictates), lanes that picked
 // the same page regroup and that page gets ONE atomicOr for all of them.
-static __device__ __noinline__ uint64_t bin_claim_collective(const ga_desc* h, unsigned grp, uint32_t A, int c) {
+static __device__ __noinline__ uint64_t bin_claim_collective(const ga_desc* h, unsigned grp, uint32_t A, int c,
+                                                             uint64_t pre_ch = 0, uint64_t pre_m = 0) {
     const uint32_t lane = lane_id();
     const uint32_t per_page = slots_of(c) < 64 ? slots_of(c) : 64;
     const uint64_t csz = 16ull << c;
@@ -1321,7 +1333,10 @@ static __device__ __noinline__ uint64_t bin_claim_collective(const ga_desc* h, u
         {
             ch = 0; m = 0;
 #endif
-            if ((int)lane == L) ch = bin_find_chunk(h, A, c, &m);
+            if ((int)lane == L) {
+                if (pre_m) { ch = pre_ch; m = pre_m; pre_m = 0; }                   // loaded beside the semaphore
+                else ch = bin_find_chunk(h, A, c, &m);
+            }
             ch = __shfl_sync(unsat, ch, L);
             m = __shfl_sync(unsat, m, L);
         }
@@ -1345,7 +1360,7 @@ static __device__ __noinline__ uint64_t bin_claim_collective(const ga_desc* h, u
                    __reduce_or_sync(unsat, (uint32_t)drop));
         }
 #endif
-        unsat = opaque_mask(__ballot_sync(unsat, my == kNull));
+        unsat = lanes_where(unsat, my == kNull);
         if (my != kNull) break;                             // a satisfied lane leaves the group
     }
     return my;
@@ -1542,45 +1557,60 @@ static __device__ __noinline__ uint64_t tree_malloc_group(const ga_desc* h, unsi
 }
 
 // ---- the entry points ---------------------------------------------------------
+// malloc.  Lanes are grouped by size class (__match_any_sync); one leader per
+// group runs Alg. 1's fetch-add for the group's N units and, in the same round
+// trip, loads the block's hinted chunk for the class (owner and non-full mask,
+// from a shared-memory hint), which the collective claim starts from.  A
+// blocked wait, growth and the per-lane fallback (R-27) run per group after it.
 static __device__ __forceinline__ uint64_t* arena_ctr(const ga_desc* h, int i) { return h->actr + arena_of(h) * kActrStride + i; }
 static __device__ __noinline__ uint64_t ga_malloc_off(const ga_desc* h, uint64_t n) {
     const unsigned act = active_lanes();
-    if ((int)lane_id() == __ffs(act) - 1) red_rlx(arena_ctr(h, 0), __popc(act));    // n_malloc, per warp
+    const uint32_t lane = lane_id();
+    if ((int)lane == __ffs(act) - 1) red_rlx(arena_ctr(h, 0), __popc(act));       // n_malloc, per warp
     const int key = size_key(h, n);
     const unsigned grp = __match_any_sync(act, key);
     if (key < 0) return kNull;
+    const int leader = __ffs(grp) - 1;
+    const uint32_t N = __popc(grp);
     uint64_t my;
     if (key < kNcls) {
         const uint32_t A = arena_of(h) / class_share(key);
-        const uint32_t N = __popc(grp), slots = slots_of(key);
-        const int leader = __ffs(grp) - 1;
-        int r = 0;
-        if ((int)lane_id() == leader) {
-            // the first fetch-add and its settling inline; a blocked wait out of line
+        const uint32_t slots = slots_of(key);
+        const uint32_t Bp = slots * ((N + slots - 1) / slots);                     // R-8
+        int r = kAcquired;
+        uint64_t w = 0, pre_ch = 0, pre_m = 0;
+        if ((int)lane == leader) {
             uint64_t* sp = sem_ptr(h, A, key);
-            const uint32_t Bp = slots * ((N + slots - 1) / slots);                     // R-8
-            uint64_t w = 0;
-            r = bsem_decide(sp, a_add(sp, dCD(-(int32_t)N, (int32_t)Bp)), N, Bp, &w);
+            const uint32_t hp = GA_PREFETCH ? s_chunk_hint[key] : 0xFFFFFFFFu;
+            const uint64_t old = a_add(sp, dCD(-(int32_t)N, (int32_t)Bp));       // Alg. 1, first fetch-add
+            uint32_t own = 0;
+            if (hp < h->pages) {                                                 // in flight with the fetch-add
+                pre_ch = hp >> kChunkShift;
+                own = ld_rlx32(&h->chunk_owner[pre_ch]);
+                pre_m = ld_rlx(nonfull_word(h, pre_ch, key));
+            }
+            r = bsem_decide(sp, old, N, Bp, &w);
             if (r == kBlocked) r = bsem_wait_slow<2048>(sp, N, Bp, ArenaSpin{h, A}, w);
+            if (own != A + 1) pre_m = 0;
         }
         r = __shfl_sync(grp, r, leader);
-        my = r == kAcquired ? bin_claim_collective(h, grp, A, key)
+        my = r == kAcquired ? bin_claim_collective(h, grp, A, key, pre_ch, pre_m)
            : is_span(key) ? span_grow_collective(h, grp, A, key) : bin_grow_collective(h, grp, A, key);
         if (__any_sync(grp, my == kNull)) {                 // R-27: degrade to per-lane waits
-            if ((int)lane_id() == leader) stat_add(h, kStatFallback, 1);
+            if ((int)lane == leader) stat_add(h, kStatFallback, 1);
             if (my == kNull) my = bin_malloc_lane(h, A, key);
         }
-    } else {
-        const int o = key - kNcls;
-        my = tree_malloc_group(h, grp, o);
-        if (my == kNull) {
-            int64_t x = tree_alloc_one_retry(h, o);
-            if (x >= 0) {
-                uint64_t pg = (uint64_t)x << o;
-                st_rlx32(&h->kind[pg], kKindTree | (uint32_t)o);
-                my = pg << kPageShift;
-            } else stat_add(h, kStatFail, 1);
-        }
+        return my;
+    }
+    const int o = key - kNcls;
+    my = tree_malloc_group(h, grp, o);
+    if (my == kNull) {
+        int64_t x = tree_alloc_one_retry(h, o);
+        if (x >= 0) {
+            uint64_t pgt = (uint64_t)x << o;
+            st_rlx32(&h->kind[pgt], kKindTree | (uint32_t)o);
+            my = pgt << kPageShift;
+        } else stat_add(h, kStatFail, 1);
     }
     return my;
 }
@@ -1596,9 +1626,9 @@ static __device__ __noinline__ void ga_free_off(const ga_desc* h, uint64_t off) 
     if (off != kNull) { p = off >> kPageShift; k = ld_rlx32(&h->kind[p]); }
     const bool is_bin = (off != kNull) && ((k & 0xC0000000u) == kKindBin);
     const bool is_tree = (off != kNull) && !is_bin;
-    const unsigned bins = opaque_mask(__ballot_sync(act, is_bin));
-    const unsigned trees = opaque_mask(__ballot_sync(act, is_tree));
-    if ((int)lane_id() == __ffs(act) - 1 && (bins | trees)) red_rlx(arena_ctr(h, 1), __popc(bins | trees));   // n_free
+    const unsigned same = __match_any_sync(act, is_bin ? 1u : is_tree ? 2u : 0u);
+    const unsigned bins = is_bin ? same : 0u, trees = is_tree ? same : 0u;      // valid in their own lanes
+    if ((int)lane_id() == __ffs(same) - 1 && (is_bin || is_tree)) red_rlx(arena_ctr(h, 1), __popc(same));   // n_free
     if (is_tree) {
         int n = (int)(k & 0xFF);                               // order from the page kind (R-18)
         uint64_t x = p >> n;
@@ -1615,7 +1645,7 @@ static __device__ __noinline__ void ga_free_off(const ga_desc* h, uint64_t off) 
                 if ((int)lane_id() == __ffs(mm) - 1) { x >>= 1; n++; }   // both halves are ours: merged
                 else alive = false;
             }
-            part = opaque_mask(__ballot_sync(part, alive));
+            part = lanes_where(part, alive);
             if (!alive) break;
         }
         if (alive) tree_free(h, n, x);
@@ -1651,7 +1681,7 @@ static __device__ __noinline__ void ga_free_off(const ga_desc* h, uint64_t off) 
     // the match is also the execution barrier: every leader's atomicAnd above
     // has returned (performed at L2) before any lane of `bins` passes it, so
     // the units signalled below never precede their slots (no __syncwarp: see
-    // opaque_mask)
+    // active_lanes)
     const unsigned g2 = __match_any_sync(bins, (A << 4) | (uint32_t)c);     // class < 16
     if ((int)lane_id() == __ffs(g2) - 1) bsem_signal_after_rmw(sem_ptr(h, A, c), __popc(g2));
     if (eager) {

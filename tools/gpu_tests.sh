@@ -7,7 +7,9 @@ mkdir -p gpurun_out
 FILES=${@:-$(ls tests/test_gpu_*.py)}
 for f in $FILES; do
   echo "== $f" >> gpurun_out/gpu_tests.log
-  timeout -k 30 ${PER_FILE_TIMEOUT:-900} python -m pytest "$f" -m gpu -q -p no:cacheprovider >> gpurun_out/gpu_tests.log 2>&1
+  # per-test timeout: a hung kernel kills this file's process after PER_TEST s
+  timeout -k 30 ${PER_FILE_TIMEOUT:-900} python -m pytest "$f" -m gpu -q -p no:cacheprovider \
+      -o timeout_func_only=false --timeout ${PER_TEST:-180} --timeout-method thread >> gpurun_out/gpu_tests.log 2>&1
   echo "rc=$? $f" >> gpurun_out/gpu_tests.log
 done
 grep -E "^== |^rc=|passed|failed|error" gpurun_out/gpu_tests.log

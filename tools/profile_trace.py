@@ -19,9 +19,11 @@ ap.add_argument("--cuda", action="store_true")
 ap.add_argument("--kmin", type=int, default=3)
 ap.add_argument("--kmax", type=int, default=15)
 ap.add_argument("--threads", type=int, default=0, help="fewer threads than the full grid (sanitizer runs)")
+ap.add_argument("--warm", action="store_true", help="no heap reset between reps")
+ap.add_argument("--level", default="pressure", help="d4 pressure level (fit / pressure / exhaust / overcommit)")
 a = ap.parse_args()
 if a.workload == "d4":
-    t = tracegen.d4_mixed("pressure", R=a.rounds)
+    t = tracegen.d4_mixed(a.level, R=a.rounds)
     if (a.kmin, a.kmax) != (3, 15):
         t = tracegen.Trace("d4_sub", tracegen.mixed_sizes(t.seed, a.rounds, t.T, a.kmin, a.kmax), 1, t.heap_bytes, t.seed)
 else:
@@ -36,6 +38,8 @@ if a.cuda:
 d = torch.from_numpy(t.sizes.view(np.int32)).cuda()
 c = torch.zeros(8, dtype=torch.int64, device="cuda")
 for i in range(a.reps):
+    if heap is not None and not a.warm:
+        heap.reset()                                   # cold heap per rep, as bench.py times it
     s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     s.record()
     run_timed(heap, d, t.R, t.T, t.D, c)
