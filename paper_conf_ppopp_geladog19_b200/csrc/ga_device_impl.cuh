@@ -609,9 +609,13 @@ static __device__ __noinline__ void tree_free(const ga_desc* h, int n, uint64_t 
 // At true exhaustion both are false.  Growth also counts other failing
 // climbers' transient E, so only the first retries may wait on it.
 static __device__ __noinline__ bool tree_has_supply(const ga_desc* h, int o, bool count_growth) {
-    for (int k = o; k <= (int)h->L; k++) {
-        uint64_t w = ld_rlx(tsem_ptr(h, k));
-        if (sem_C(w) >= 1 || (count_growth && sem_D(w) > 0)) return true;
+    for (int k0 = o; k0 <= (int)h->L; k0 += 8) {                 // 8 independent loads per round trip
+        uint64_t w[8];
+#pragma unroll
+        for (int i = 0; i < 8; i++) w[i] = k0 + i <= (int)h->L ? ld_rlx(tsem_ptr(h, k0 + i)) : dCD(0, 0);
+#pragma unroll
+        for (int i = 0; i < 8; i++)
+            if (sem_C(w[i]) >= 1 || (count_growth && sem_D(w[i]) > 0)) return true;
     }
     return false;
 }
@@ -700,9 +704,9 @@ static __device__ __noinline__ void nonfull_clear_if_full(const ga_desc* h, uint
 }
 
 // Take a new chunk from TBuddy for arena A, keep its first k pages, open the rest.
-static __device__ __noinline__ int64_t tree_alloc_one_retry(const ga_desc* h, int o);
+static __device__ __noinline__ int64_t tree_alloc_one_retry(const ga_desc* h, int o, bool chunk_supply);
 static __device__ __noinline__ int64_t chunk_acquire(const ga_desc* h, uint32_t A, uint32_t k) {
-    int64_t ch = tree_alloc_one_retry(h, kChunkOrder);
+    int64_t ch = tree_alloc_one_retry(h, kChunkOrder, true);
     if (ch < 0) return -1;
     st_rlx32(&h->chunk_owner[ch], A + 1);
     fence();
@@ -1161,17 +1165,40 @@ static __device__ __noinline__ int reclaim_arena(const ga_desc* h, uint32_t A, i
     }
     return done;
 }
-static __device__ __noinline__ void reclaim_all(const ga_desc* h) {
-    for (uint32_t A = 0; A < h->n_arenas; A++) reclaim_arena(h, A, -1, 0);
+// Reclaim every candidate of arenas A0, A0 + step, ...: the arenas' top summary
+// words are loaded 16 at a time (independent loads, one round trip per batch)
+// and only arenas with candidates are visited.
+static __device__ __noinline__ void reclaim_arenas(const ga_desc* h, uint32_t A0, uint32_t step) {
+    for (uint32_t base = A0; base < h->n_arenas; base += 16 * step) {
+        uint64_t top[16];
+#pragma unroll
+        for (int i = 0; i < 16; i++) {
+            const uint32_t A = base + i * step;
+            top[i] = A < h->n_arenas ? ld_rlx(hb3_w2(arena_hb(h, A, kAhbCnd))) : 0;
+        }
+#pragma unroll 1
+        for (int i = 0; i < 16; i++)
+            if (top[i]) reclaim_arena(h, base + i * step, -1, 0);
+    }
 }
+static __device__ __noinline__ void reclaim_all(const ga_desc* h) { reclaim_arenas(h, 0, 1); }
 
 // Per-lane TBuddy allocation with the no-false-starvation retry: the optimistic
 // order semaphores can send a lane up the tree while another lane's split is
 // still in flight.  Retry while the tree shows supply; drain reclamation once.
-static __device__ __noinline__ int64_t tree_alloc_one_retry(const ga_desc* h, int o) {
+// chunk_supply: the caller is a bin / span grower whose failure the arena
+// fallback (group_fallback) re-checks against growth in flight, so it fails
+// at once when no order >= o holds an Available node (other climbers' expected
+// units at exhaustion are failing climbers, and waiting on them convoys).
+static __device__ __noinline__ int64_t tree_alloc_one_retry(const ga_desc* h, int o, bool chunk_supply) {
     GA_DBG_CNT;
     bool drained = false;
     uint32_t ns = 64;
+    if (chunk_supply && !tree_has_supply(h, o, false)) {   // nothing Available at any order >= o:
+        reclaim_all(h);                                     // drain once, and climb only if that freed something
+        if (!tree_has_supply(h, o, false)) return -1;
+        drained = true;
+    }
     for (int attempt = 0; attempt < 32; attempt++) {
         int64_t x = tree_alloc_one(h, o);
         if (x >= 0) return x;
@@ -1218,7 +1245,7 @@ static __device__ __noinline__ uint64_t bin_claim_one(const ga_desc* h, uint32_t
 }
 // a fresh span for arena A straight from TBuddy (one chunk); -1 if the tree is exhausted
 static __device__ __noinline__ int64_t span_acquire(const ga_desc* h, uint32_t A) {
-    int64_t ch = tree_alloc_one_retry(h, kChunkOrder);
+    int64_t ch = tree_alloc_one_retry(h, kChunkOrder, true);
     if (ch < 0) return -1;
     st_rlx32(&h->chunk_owner[ch], A + 1);
     stat_add(h, kStatChunkGrow, 1);
@@ -1556,13 +1583,109 @@ static __device__ __noinline__ uint64_t tree_malloc_group(const ga_desc* h, unsi
     return my;
 }
 
+// ---- malloc of a bin / span class in one arena, and the group fallback --------
+static __device__ __forceinline__ uint64_t* arena_ctr(const ga_desc* h, int i) { return h->actr + arena_of(h) * kActrStride + i; }
+// malloc of class c (bin or span) for the lanes of grp in arena A: Alg. 1 wait,
+// then the collective claim or growth.  Lanes it could not serve get kNull.
+// pre_ch / pre_m: a chunk and its non-full mask the leader loaded beside the
+// fetch-add (pre_m == 0: none).
+static __device__ __forceinline__ uint64_t malloc_in_arena(const ga_desc* h, unsigned grp, uint32_t A, int c,
+                                                           bool prefetch) {
+    const uint32_t lane = lane_id();
+    const int leader = __ffs(grp) - 1;
+    const uint32_t N = __popc(grp);
+    const uint32_t slots = slots_of(c);
+    const uint32_t Bp = slots * ((N + slots - 1) / slots);                         // R-8
+    int r = kAcquired;
+    uint64_t w = 0, pre_ch = 0, pre_m = 0;
+    if ((int)lane == leader) {
+        uint64_t* sp = sem_ptr(h, A, c);
+        const uint32_t hp = GA_PREFETCH && prefetch ? s_chunk_hint[c] : 0xFFFFFFFFu;
+        const uint64_t old = a_add(sp, dCD(-(int32_t)N, (int32_t)Bp));           // Alg. 1, first fetch-add
+        uint32_t own = 0;
+        if (hp < h->pages) {                                                     // in flight with the fetch-add
+            pre_ch = hp >> kChunkShift;
+            own = ld_rlx32(&h->chunk_owner[pre_ch]);
+            pre_m = ld_rlx(nonfull_word(h, pre_ch, c));
+        }
+        r = bsem_decide(sp, old, N, Bp, &w);
+        if (r == kBlocked) r = bsem_wait_slow<2048>(sp, N, Bp, ArenaSpin{h, A}, w);
+        if (own != A + 1) pre_m = 0;
+    }
+    r = __shfl_sync(grp, r, leader);
+    return r == kAcquired ? bin_claim_collective(h, grp, A, c, pre_ch, pre_m)
+         : is_span(c) ? span_grow_collective(h, grp, A, c) : bin_grow_collective(h, grp, A, c);
+}
+
+// The group-level fallback (R-26: a malloc fails only if no arena
+// can serve it).  The group's own arena could not grow (the tree is empty).
+// Delegated reclamation is drained once, then the group's lanes scan every
+// arena's class and page semaphores in parallel (one load each per lane) and
+// take the richest arena, where the group runs the normal sequence; repeat for
+// the lanes still unserved.  When no arena shows units, pages or a growth in
+// flight and the tree has no chunk, the group fails at once -- no per-lane
+// scans.  A group that keeps missing for other reasons ends in the exact
+// per-lane path (bin_malloc_lane).
+static __device__ __noinline__ uint64_t group_fallback(const ga_desc* h, unsigned grp, uint32_t A0, int c) {
+    const uint32_t lane = lane_id();
+    reclaim_arenas(h, __popc(grp & lanemask_lt()), __popc(grp));                 // P:L1206-1244, lanes in parallel
+    (void)__shfl_sync(grp, 0, __ffs(grp) - 1);
+    const bool span = is_span(c);
+    const uint32_t nA = (h->n_arenas + class_share(c) - 1) / class_share(c);     // arenas of class c
+    uint64_t my = kNull;
+    unsigned rest = grp;
+    bool seen_nothing = false;
+    for (int tries = 0; tries < 32; tries++) {
+        const uint32_t n = __popc(rest), q = __popc(rest & lanemask_lt());
+        const int L = __ffs(rest) - 1;
+        uint32_t best = 0;                                                       // units << 8 | arena
+        for (uint32_t B = q; B < nA; B += n) {
+            const uint64_t sw = ld_rlx(sem_ptr(h, B, c));
+            int64_t units = sem_C(sw) > 0 ? sem_C(sw) : 0;
+            if (!span) {
+                const uint64_t pw = ld_rlx(psem_ptr(h, B));
+                units += (int64_t)(sem_C(pw) > 0 ? sem_C(pw) : 0) * slots_of(c);
+            }
+            const uint32_t pk = ((uint32_t)(units < 0xFFFFFF ? units : 0xFFFFFF) << 8) | B;
+            best = pk > best ? pk : best;
+        }
+        best = __reduce_max_sync(rest, best);
+        uint32_t target;
+        if (best >> 8) {
+            target = best & 0xFF;                                                // an arena with units or pages
+        } else {
+            // No arena shows units or pages.  The tree may still supply a chunk
+            // (grow at home), or a split may be publishing one (count_growth).
+            int t = 0;
+            if ((int)lane == L) t = tree_has_supply(h, kChunkOrder, false) ? 2 : tree_has_supply(h, kChunkOrder, true) ? 1 : 0;
+            t = __shfl_sync(rest, t, L);
+            if (t == 2) target = A0;
+            else if (t == 1 || !seen_nothing) {
+                // a split in flight, or a grower that already holds its pages and
+                // is about to publish: look again once it had time to finish
+                seen_nothing = t == 0;
+                __nanosleep(8192);
+                continue;
+            } else {
+                if ((int)lane == L) stat_add(h, kStatFail, __popc(rest));
+                return kNull;                                                    // nothing anywhere: fail
+            }
+        }
+        seen_nothing = false;
+        my = malloc_in_arena(h, rest, target, c, false);
+        rest = lanes_where(rest, my == kNull);
+        if (my != kNull) return my;
+    }
+    // still unserved after many rounds: the exact per-lane path (R-26, R-27)
+    return bin_malloc_lane(h, A0, c);
+}
+
 // ---- the entry points ---------------------------------------------------------
 // malloc.  Lanes are grouped by size class (__match_any_sync); one leader per
 // group runs Alg. 1's fetch-add for the group's N units and, in the same round
 // trip, loads the block's hinted chunk for the class (owner and non-full mask,
-// from a shared-memory hint), which the collective claim starts from.  A
-// blocked wait, growth and the per-lane fallback (R-27) run per group after it.
-static __device__ __forceinline__ uint64_t* arena_ctr(const ga_desc* h, int i) { return h->actr + arena_of(h) * kActrStride + i; }
+// from a shared-memory hint), which the collective claim starts from.  Lanes
+// the arena cannot serve take the group fallback (R-26, R-27).
 static __device__ __noinline__ uint64_t ga_malloc_off(const ga_desc* h, uint64_t n) {
     const unsigned act = active_lanes();
     const uint32_t lane = lane_id();
@@ -1570,42 +1693,21 @@ static __device__ __noinline__ uint64_t ga_malloc_off(const ga_desc* h, uint64_t
     const int key = size_key(h, n);
     const unsigned grp = __match_any_sync(act, key);
     if (key < 0) return kNull;
-    const int leader = __ffs(grp) - 1;
-    const uint32_t N = __popc(grp);
     uint64_t my;
     if (key < kNcls) {
         const uint32_t A = arena_of(h) / class_share(key);
-        const uint32_t slots = slots_of(key);
-        const uint32_t Bp = slots * ((N + slots - 1) / slots);                     // R-8
-        int r = kAcquired;
-        uint64_t w = 0, pre_ch = 0, pre_m = 0;
-        if ((int)lane == leader) {
-            uint64_t* sp = sem_ptr(h, A, key);
-            const uint32_t hp = GA_PREFETCH ? s_chunk_hint[key] : 0xFFFFFFFFu;
-            const uint64_t old = a_add(sp, dCD(-(int32_t)N, (int32_t)Bp));       // Alg. 1, first fetch-add
-            uint32_t own = 0;
-            if (hp < h->pages) {                                                 // in flight with the fetch-add
-                pre_ch = hp >> kChunkShift;
-                own = ld_rlx32(&h->chunk_owner[pre_ch]);
-                pre_m = ld_rlx(nonfull_word(h, pre_ch, key));
-            }
-            r = bsem_decide(sp, old, N, Bp, &w);
-            if (r == kBlocked) r = bsem_wait_slow<2048>(sp, N, Bp, ArenaSpin{h, A}, w);
-            if (own != A + 1) pre_m = 0;
-        }
-        r = __shfl_sync(grp, r, leader);
-        my = r == kAcquired ? bin_claim_collective(h, grp, A, key, pre_ch, pre_m)
-           : is_span(key) ? span_grow_collective(h, grp, A, key) : bin_grow_collective(h, grp, A, key);
-        if (__any_sync(grp, my == kNull)) {                 // R-27: degrade to per-lane waits
-            if ((int)lane == leader) stat_add(h, kStatFallback, 1);
-            if (my == kNull) my = bin_malloc_lane(h, A, key);
+        my = malloc_in_arena(h, grp, A, key, true);
+        if (__any_sync(grp, my == kNull)) {
+            const unsigned rest = lanes_where(grp, my == kNull);
+            if ((int)lane == __ffs(grp) - 1) stat_add(h, kStatFallback, 1);
+            if (my == kNull) my = group_fallback(h, rest, A, key);
         }
         return my;
     }
     const int o = key - kNcls;
     my = tree_malloc_group(h, grp, o);
     if (my == kNull) {
-        int64_t x = tree_alloc_one_retry(h, o);
+        int64_t x = tree_alloc_one_retry(h, o, false);
         if (x >= 0) {
             uint64_t pgt = (uint64_t)x << o;
             st_rlx32(&h->kind[pgt], kKindTree | (uint32_t)o);
