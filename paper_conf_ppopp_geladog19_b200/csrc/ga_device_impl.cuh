@@ -1464,6 +1464,7 @@ static __device__ __noinline__ uint64_t bin_grow_collective(const ga_desc* h, un
 // them initialises the span.  If the tree runs dry the lanes served so far
 // keep their slots, the others get kNull (the caller degrades them to per-lane
 // waits) and the unproduced units are retracted (signal(0, B'-N)).
+static __device__ __noinline__ uint64_t tree_malloc_group(const ga_desc* h, unsigned grp, int o);
 static __device__ __noinline__ uint64_t span_grow_collective(const ga_desc* h, unsigned grp, uint32_t A, int c) {
     const uint32_t lane = lane_id();
     const int leader = __ffs(grp) - 1;
@@ -1472,13 +1473,43 @@ static __device__ __noinline__ uint64_t span_grow_collective(const ga_desc* h, u
     const uint32_t Bp = slots * ((N + slots - 1) / slots);                 // R-8
     const uint64_t csz = 16ull << c;
     uint64_t my = kNull;
+    const uint32_t k = Bp / slots;
+    if ((int)lane == leader) reclaim_arena(h, A, -1, kReclaimKeep);           // delegated work first
+    if (k > 1) {
+        // All k chunks in ONE collective TBuddy claim (tree_malloc_group: one
+        // semaphore wait per level and up to 64 nodes per bitmap atomic, the
+        // collective critical section of) instead of k climbs.
+        // All-or-nothing: if the tree cannot serve k at once nothing was taken
+        // and the chunk-at-a-time loop below runs.
+        const unsigned sub = lanes_where(grp, rank < k);
+        int64_t mych = -1;
+        if (rank < k) {
+            const uint64_t off = tree_malloc_group(h, sub, kChunkOrder);
+            if (off != kNull) {
+                mych = (int64_t)(off >> (kPageShift + kChunkShift));
+                st_rlx32(&h->chunk_owner[mych], A + 1);
+                stat_add(h, kStatChunkGrow, 1);
+            }
+        }
+        if (__all_sync(grp, rank >= k || mych >= 0)) {
+            const uint32_t j = rank / slots, r = rank % slots;
+            const int64_t chj = __shfl_sync(grp, mych, (int)nth_set(grp, j));    // span j: the j-th lane's chunk
+            const uint64_t p = (uint64_t)chj * kChunkPages;
+            my = (p << kPageShift) + (uint64_t)r * csz;
+            if (r == 0) bin_init(h, p, A, c, N - j * slots < slots ? N - j * slots : slots);
+            warp_release(grp);
+            if ((int)lane == leader) {
+                stat_add(h, kStatBinGrow, k);
+                st_rlx32(&h->hint[A * kNcls + c], (uint32_t)p);
+                bsem_signal(sem_ptr(h, A, c), Bp - N, Bp - N);                  // release: spans initialised
+            }
+            return my;
+        }
+    }
     uint32_t served = 0;
     int64_t ch = 0;
     while (served < N) {
-        if ((int)lane == leader) {
-            if (served == 0) reclaim_arena(h, A, -1, kReclaimKeep);       // delegated work first
-            ch = span_acquire(h, A);
-        }
+        if ((int)lane == leader) ch = span_acquire(h, A);
         ch = __shfl_sync(grp, ch, leader);
         if (ch < 0) break;
         const uint32_t take = N - served < slots ? N - served : slots;
