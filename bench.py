@@ -39,18 +39,20 @@ L2_FLUSH_BYTES = 512 << 20
 
 
 # ----------------------------------------------------------------------------- helpers
-def algorithmic_atomics(sizes: np.ndarray) -> int:
+def algorithmic_atomics(sizes: np.ndarray, group: int = 32) -> int:
     """Minimum L2 atomics the method must issue for one pass of a D=1 trace with
     every call succeeding: per warp-round and size class,
     a group of N lanes needs 1 semaphore op + ceil(N / slots-per-bitmap-word)
     tracking ops (bins: min(64, 4096/class); tree: 64 nodes per level word), for
-    the mallocs and again for the frees of the same blocks."""
+    the mallocs and again for the frees of the same blocks.  `group`: threads
+    that call together (32 warp calls; the block or cluster size for the
+    collective calls, whose class groups are whole CTAs / clusters)."""
     R, T = sizes.shape
     n = sizes.astype(np.int64)
     lg = np.ceil(np.log2(np.maximum(n, 16))).astype(np.int64)           # class log2
     key = lg - 4                                                        # 0..7 bins, 8.. tree
-    W = T // 32
-    k = key[:, : W * 32].reshape(R, W, 32)
+    W = T // group
+    k = key[:, : W * group].reshape(R, W, group)
     total = 0
     for c in range(int(key.max()) + 1):
         N = (k == c).sum(axis=2)

@@ -35,6 +35,17 @@ typedef struct { uint64_t off; uint32_t size; uint32_t meta; } ga_log_rec;
 
 enum { GA_TRACE_LOG = 1, GA_TRACE_TAG = 2 };
 
+/* Scope of the allocator calls a trace kernel makes (flags bits 8..11 of
+ * ga_trace_phase, `scope` of ga_trace_timed_scope):
+ *   0     -- warp path: ga_malloc / ga_free (include/ga_device.cuh);
+ *   1     -- block-collective: ga_malloc_block / ga_free_block;
+ *   2..8  -- cluster-collective over clusters of that many CTAs:
+ *            ga_malloc_cluster / ga_free_cluster (the grid is padded to a
+ *            multiple of the cluster; block * cluster <= 2048).
+ * Collective kernels keep every thread in every call (threads past T pass
+ * n == 0 / NULL).  Invalid scopes return GA_EINVAL. */
+#define GA_TRACE_SCOPE(s) ((uint32_t)(s) << 8)
+
 /* Correctness mode: one kernel per phase.  held: DEVICE u64[2*T] (block, size),
  * all ~0 / 0 before round 0.  D == 1: round in [0, R], phase ignored.
  * D == 0: round in [0, R), phase 0 = malloc, 1 = free. */
@@ -46,6 +57,11 @@ ga_status ga_trace_phase(ga_heap_t h, ga_stream_t stream, const uint32_t* sizes,
  * no tags and no extra memory traffic: the allocator alone. */
 ga_status ga_trace_timed(ga_heap_t h, ga_stream_t stream, const uint32_t* sizes, uint32_t R,
                          uint32_t T, uint32_t D, uint64_t* counts, uint32_t block);
+
+/* ga_trace_timed with the calls at `scope` (see GA_TRACE_SCOPE; 0 is
+ * ga_trace_timed itself). */
+ga_status ga_trace_timed_scope(ga_heap_t h, ga_stream_t stream, const uint32_t* sizes, uint32_t R,
+                               uint32_t T, uint32_t D, uint64_t* counts, uint32_t block, uint32_t scope);
 
 /* End-to-end: HOST sizes (pinned for overlap) copied H2D, the timed kernel,
  * counts copied D2H into host u64[4]; synchronises `stream`.  Scratch device

@@ -9,7 +9,9 @@
  * full-occupancy grid, from converged or divergent code.
  *
  * ga_malloc: rounds n up to a power of two >= 16 B (R-13, R-14); 16..2048 B
- *   come from one-page bins (UAlloc), larger sizes from TBuddy
+ *   come from one-page bins (UAlloc), 4..64 KiB from "spans" (one
+ *   64-page chunk split into 64..4 slots, served like bins; DESIGN.md section 7;
+ *   GA_NSPAN=0 restores the paper's routing), larger sizes from TBuddy
  *   (P:L834-1016).  Returns a pointer aligned to its class (bins) or its block
  *   size (TBuddy, relative to the 2 MiB aligned base, R-31), or NULL when n == 0,
  *   n exceeds the heap, or no arena can serve the request after every fallback
@@ -43,6 +45,38 @@ __device__ __forceinline__ void* ga_malloc(ga_dev_heap h, size_t n) {
 
 __device__ __forceinline__ void ga_free(ga_dev_heap h, void* p) {
     ga::ga_free_off(h.desc, p ? (uint64_t)((char*)p - h.base) : ga::kNull);
+}
+
+/* Block- and cluster-collective calls (the paper's collective synchronization
+ * primitives at thread-block scope, Sec. 4.2.2; cluster scope
+ * through distributed shared memory is the B200 extension).
+ *
+ * EVERY thread of the CTA (ga_*_block) or of the thread-block cluster
+ * (ga_*_cluster) must make the same sequence of calls, like __syncthreads();
+ * threads with nothing to do pass n == 0 / p == NULL.  Each call contains one
+ * (free) or two (malloc) barriers of that scope.  Call ga_block_begin /
+ * ga_cluster_begin once per kernel, by every thread, before the first call.
+ * A block or cluster call serves at most 2048 threads.  Per class, ONE thread
+ * performs the semaphore operation for the whole collective's demand, and the
+ * released units of a collective free reach the semaphores as one signal per
+ * class.  Sizes above 64 KiB (TBuddy) take the warp path inside the call.
+ * The static shared state (~170 B per CTA) is only allocated in kernels that
+ * use these calls.  Same results and failure rules as ga_malloc/ga_free. */
+__device__ __forceinline__ void ga_block_begin(ga_dev_heap h) { ga::coll_begin<false>(h.desc); }
+__device__ __forceinline__ void* ga_malloc_block(ga_dev_heap h, size_t n) {
+    uint64_t off = ga::malloc_coll_off<false>(h.desc, (uint64_t)n);
+    return off == ga::kNull ? nullptr : (void*)(h.base + off);
+}
+__device__ __forceinline__ void ga_free_block(ga_dev_heap h, void* p) {
+    ga::free_coll_off<false>(h.desc, p ? (uint64_t)((char*)p - h.base) : ga::kNull);
+}
+__device__ __forceinline__ void ga_cluster_begin(ga_dev_heap h) { ga::coll_begin<true>(h.desc); }
+__device__ __forceinline__ void* ga_malloc_cluster(ga_dev_heap h, size_t n) {
+    uint64_t off = ga::malloc_coll_off<true>(h.desc, (uint64_t)n);
+    return off == ga::kNull ? nullptr : (void*)(h.base + off);
+}
+__device__ __forceinline__ void ga_free_cluster(ga_dev_heap h, void* p) {
+    ga::free_coll_off<true>(h.desc, p ? (uint64_t)((char*)p - h.base) : ga::kNull);
 }
 
 /* Bulk-semaphore primitives (Alg. 1 / Alg. 2), exported for the

@@ -16,7 +16,8 @@ from . import _build
 __all__ = ["lib", "GaError", "Layout", "Stats", "DevHeap", "ga_heap_create", "ga_heap_destroy",
            "ga_heap_reset", "ga_stats", "ga_heap_device", "ga_heap_info", "ga_layout",
            "ga_heap_quiesce", "ga_heap_snapshot", "ga_reserved_pages", "ga_status_str",
-           "ga_trace_phase", "ga_trace_timed", "ga_trace_timed_host", "ga_cuda_set_heap_limit",
+           "ga_trace_phase", "ga_trace_timed", "ga_trace_timed_scope", "ga_trace_timed_host",
+           "ga_cuda_set_heap_limit", "GA_TRACE_SCOPE",
            "ga_cuda_trace_phase", "ga_cuda_trace_timed", "ga_kernel_info", "ga_l2_atomic_bench",
            "ga_bsem_bench", "BsemCfg", "EXPORTED", "GA_TRACE_LOG", "GA_TRACE_TAG",
            "ga_rcu_workspace_bytes", "ga_rcu_list_removal", "ga_edge_calls"]
@@ -24,10 +25,15 @@ __all__ = ["lib", "GaError", "Layout", "Stats", "DevHeap", "ga_heap_create", "ga
 GA_TRACE_LOG = 1
 GA_TRACE_TAG = 2
 
+
+def GA_TRACE_SCOPE(scope: int) -> int:
+    """flags bits 8..11: 0 warp calls, 1 block-collective, 2..8 cluster-collective (include/ga_bench.h)"""
+    return scope << 8
+
 # every symbol include/ga.h and include/ga_bench.h declare
 EXPORTED = ["ga_heap_create", "ga_heap_destroy", "ga_heap_reset", "ga_stats", "ga_heap_device",
             "ga_heap_info", "ga_layout", "ga_heap_quiesce", "ga_heap_snapshot", "ga_reserved_pages",
-            "ga_status_str", "ga_trace_phase", "ga_trace_timed", "ga_trace_timed_host",
+            "ga_status_str", "ga_trace_phase", "ga_trace_timed", "ga_trace_timed_scope", "ga_trace_timed_host",
             "ga_cuda_set_heap_limit", "ga_cuda_trace_phase", "ga_cuda_trace_timed",
             "ga_kernel_info", "ga_l2_atomic_bench", "ga_bsem_bench", "ga_debug_attach", "ga_edge_calls",
             "ga_rcu_workspace_bytes", "ga_rcu_list_removal"]
@@ -91,6 +97,7 @@ def lib():
         "ga_reserved_pages": [vp, vp, P(u64)],
         "ga_trace_phase": [vp, vp, vp, u32, u32, u32, u32, u32, vp, vp, vp, u32, u32],
         "ga_trace_timed": [vp, vp, vp, u32, u32, u32, vp, u32],
+        "ga_trace_timed_scope": [vp, vp, vp, u32, u32, u32, vp, u32, u32],
         "ga_trace_timed_host": [vp, vp, vp, u32, u32, u32, vp, u32],
         "ga_cuda_set_heap_limit": [sz],
         "ga_cuda_trace_phase": [vp, vp, u32, u32, u32, u32, u32, vp, vp, u32, u32],
@@ -186,6 +193,10 @@ def ga_trace_phase(h, stream, sizes, R, T, D, rnd, phase, held, log, counts, fla
 
 def ga_trace_timed(h, stream, sizes, R, T, D, counts, block=256):
     _ok(lib().ga_trace_timed(h, stream or None, sizes, R, T, D, counts, block), "ga_trace_timed")
+
+
+def ga_trace_timed_scope(h, stream, sizes, R, T, D, counts, block=256, scope=0):
+    _ok(lib().ga_trace_timed_scope(h, stream or None, sizes, R, T, D, counts, block, scope), "ga_trace_timed_scope")
 
 
 def ga_trace_timed_host(h, stream, host_sizes, R, T, D, host_counts, block=256):

@@ -30,13 +30,36 @@ namespace {
 constexpr uint64_t kNullOff = ~0ull;
 
 struct GaPolicy {
+    static constexpr bool kColl = false;
     ga_dev_heap h;      // 16-byte handle: descriptor pointer + base
+    __device__ void begin() const {}
     __device__ void* alloc(uint64_t n) const { return ga_malloc(h, n); }
     __device__ void release(void* p) const { ga_free(h, p); }
     __device__ uint64_t off(const void* p) const { return p ? (uint64_t)((const char*)p - h.base) : kNullOff; }
     __device__ void* ptr(uint64_t o) const { return o == kNullOff ? nullptr : (void*)(h.base + o); }
 };
+// block- / cluster-collective calls: every thread of the CTA / cluster calls
+struct GaBlockPolicy {
+    static constexpr bool kColl = true;
+    ga_dev_heap h;
+    __device__ void begin() const { ga_block_begin(h); }
+    __device__ void* alloc(uint64_t n) const { return ga_malloc_block(h, n); }
+    __device__ void release(void* p) const { ga_free_block(h, p); }
+    __device__ uint64_t off(const void* p) const { return p ? (uint64_t)((const char*)p - h.base) : kNullOff; }
+    __device__ void* ptr(uint64_t o) const { return o == kNullOff ? nullptr : (void*)(h.base + o); }
+};
+struct GaClusterPolicy {
+    static constexpr bool kColl = true;
+    ga_dev_heap h;
+    __device__ void begin() const { ga_cluster_begin(h); }
+    __device__ void* alloc(uint64_t n) const { return ga_malloc_cluster(h, n); }
+    __device__ void release(void* p) const { ga_free_cluster(h, p); }
+    __device__ uint64_t off(const void* p) const { return p ? (uint64_t)((const char*)p - h.base) : kNullOff; }
+    __device__ void* ptr(uint64_t o) const { return o == kNullOff ? nullptr : (void*)(h.base + o); }
+};
 struct CudaPolicy {
+    static constexpr bool kColl = false;
+    __device__ void begin() const {}
     __device__ void* alloc(uint64_t n) const { return malloc(n); }
     __device__ void release(void* p) const { free(p); }
     __device__ uint64_t off(const void* p) const { return p ? (uint64_t)p : kNullOff; }
@@ -75,25 +98,31 @@ __device__ __forceinline__ void flush_counts(uint64_t* counts, uint32_t nm, uint
     }
 }
 
-// D == 1 correctness round r in [0, R]: free the held block, then malloc (r < R)
+// D == 1 correctness round r in [0, R]: free the held block, then malloc (r < R).
+// Collective policies keep threads t >= T in every call (free NULL, malloc 0).
 template <class P>
 __global__ void __launch_bounds__(256) k_churn_round(P al, const uint32_t* sizes, uint32_t R, uint32_t T, uint32_t r,
                                                      uint64_t* held, ga_log_rec* log, uint64_t* counts, uint32_t flags) {
     uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
-    if (t >= T) return;
+    if (!P::kColl && t >= T) return;
+    const bool live = t < T;
+    al.begin();
     uint32_t nm = 0, nf = 0, nfree = 0, nbad = 0;
     uint64_t idx = 2ull * ((uint64_t)r * T + t);
-    uint64_t hp = held[2 * t];
-    uint32_t hs = (uint32_t)held[2 * t + 1];
+    uint64_t hp = live ? held[2 * t] : kNullOff;
+    uint32_t hs = live ? (uint32_t)held[2 * t + 1] : 0;
     if (hp != kNullOff) {
         void* p = al.ptr(hp);
         if ((flags & GA_TRACE_TAG) && !tag_ok(p, hs, tag_of(t, r - 1))) nbad++;
         al.release(p);
         nfree++;
         logw(log, idx + 1, hp, hs, meta_of(t, r, 1));
-    } else logw(log, idx + 1, kNullOff, 0, 0);
+    } else {
+        if (P::kColl) al.release(nullptr);
+        if (live) logw(log, idx + 1, kNullOff, 0, 0);
+    }
     hp = kNullOff; hs = 0;
-    uint32_t n = r < R ? sizes[(uint64_t)r * T + t] : 0;
+    uint32_t n = r < R && live ? sizes[(uint64_t)r * T + t] : 0;
     if (n) {
         void* p = al.alloc(n);
         nm++;
@@ -103,9 +132,14 @@ __global__ void __launch_bounds__(256) k_churn_round(P al, const uint32_t* sizes
             hp = al.off(p); hs = n;
         }
         logw(log, idx, al.off(p), n, meta_of(t, r, 0));
-    } else logw(log, idx, kNullOff, 0, 0);
-    held[2 * t] = hp;
-    held[2 * t + 1] = hs;
+    } else {
+        if (P::kColl) al.alloc(0);
+        if (live) logw(log, idx, kNullOff, 0, 0);
+    }
+    if (live) {
+        held[2 * t] = hp;
+        held[2 * t + 1] = hs;
+    }
     flush_counts(counts, nm, nf, nfree, nbad);
 }
 
@@ -114,11 +148,13 @@ template <class P>
 __global__ void __launch_bounds__(256) k_phase(P al, const uint32_t* sizes, uint32_t T, uint32_t r, uint32_t phase,
                                                uint64_t* held, ga_log_rec* log, uint64_t* counts, uint32_t flags) {
     uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
-    if (t >= T) return;
+    if (!P::kColl && t >= T) return;
+    const bool live = t < T;
+    al.begin();
     uint32_t nm = 0, nf = 0, nfree = 0, nbad = 0;
     uint64_t idx = 2ull * ((uint64_t)r * T + t);
     if (phase == 0) {
-        uint32_t n = sizes[(uint64_t)r * T + t];
+        uint32_t n = live ? sizes[(uint64_t)r * T + t] : 0;
         uint64_t hp = kNullOff;
         if (n) {
             void* p = al.alloc(n);
@@ -126,21 +162,31 @@ __global__ void __launch_bounds__(256) k_phase(P al, const uint32_t* sizes, uint
             if (!p) nf++;
             else { if (flags & GA_TRACE_TAG) tag_write(p, n, tag_of(t, r)); hp = al.off(p); }
             logw(log, idx, al.off(p), n, meta_of(t, r, 0));
-        } else logw(log, idx, kNullOff, 0, 0);
-        held[2 * t] = hp;
-        held[2 * t + 1] = hp == kNullOff ? 0 : n;
+        } else {
+            if (P::kColl) al.alloc(0);
+            if (live) logw(log, idx, kNullOff, 0, 0);
+        }
+        if (live) {
+            held[2 * t] = hp;
+            held[2 * t + 1] = hp == kNullOff ? 0 : n;
+        }
     } else {
-        uint64_t hp = held[2 * t];
-        uint32_t hs = (uint32_t)held[2 * t + 1];
+        uint64_t hp = live ? held[2 * t] : kNullOff;
+        uint32_t hs = live ? (uint32_t)held[2 * t + 1] : 0;
         if (hp != kNullOff) {
             void* p = al.ptr(hp);
             if ((flags & GA_TRACE_TAG) && !tag_ok(p, hs, tag_of(t, r))) nbad++;
             al.release(p);
             nfree++;
             logw(log, idx + 1, hp, hs, meta_of(t, r, 1));
-        } else logw(log, idx + 1, kNullOff, 0, 0);
-        held[2 * t] = kNullOff;
-        held[2 * t + 1] = 0;
+        } else {
+            if (P::kColl) al.release(nullptr);
+            if (live) logw(log, idx + 1, kNullOff, 0, 0);
+        }
+        if (live) {
+            held[2 * t] = kNullOff;
+            held[2 * t + 1] = 0;
+        }
     }
     flush_counts(counts, nm, nf, nfree, nbad);
 }
@@ -150,11 +196,27 @@ template <class P, int MINB>
 __global__ void __launch_bounds__(256, MINB) k_timed(P al, const uint32_t* __restrict__ sizes, uint32_t R, uint32_t T, uint32_t D,
                                                uint64_t* counts) {
     uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
-    if (t >= T) return;
+    if (!P::kColl && t >= T) return;
+    const bool live = t < T;
+    al.begin();
     uint32_t nm = 0, nf = 0, nfree = 0;
     void* held = nullptr;
     for (uint32_t r = 0; r < R; r++) {
-        uint32_t n = __ldg(&sizes[(uint64_t)r * T + t]);
+        uint32_t n = live ? __ldg(&sizes[(uint64_t)r * T + t]) : 0;
+        if (P::kColl) {
+            // collective calls: every thread, every call (the barriers inside reconverge)
+            if (D) {
+                if (held) nfree++;
+                al.release(held);
+                held = al.alloc(n);
+                if (n) { nm++; nf += held == nullptr; }
+            } else {
+                void* p = al.alloc(n);
+                if (n) { nm++; if (p) nfree++; else nf++; }
+                al.release(p);
+            }
+            continue;
+        }
 #if GA_TIMED_SYNCWARP
         // reconverge the warp before each call, as a user kernel calling from
         // converged code would (T % 32 == 0: every warp runs every round whole)
@@ -172,7 +234,8 @@ __global__ void __launch_bounds__(256, MINB) k_timed(P al, const uint32_t* __res
             if (p) { al.release(p); nfree++; } else nf++;
         }
     }
-    if (held) { al.release(held); nfree++; }
+    if (P::kColl) { if (held) nfree++; al.release(held); }
+    else if (held) { al.release(held); nfree++; }
     flush_counts(counts, nm, nf, nfree, 0);
 }
 
@@ -333,6 +396,30 @@ inline int occupancy_target() {
 inline uint32_t nblocks(uint32_t T, uint32_t block) { return (T + block - 1) / block; }
 inline ga_status launched() { return cudaGetLastError() == cudaSuccess ? GA_OK : GA_ECUDA; }
 
+// scope of the calls (GA_TRACE_SCOPE): 0 warp, 1 block, 2..8 cluster size
+inline bool scope_ok(uint32_t scope, uint32_t block) {
+    if (scope > 8) return false;
+    return scope == 0 || block * (scope > 1 ? scope : 1) <= ga::kCollMax;
+}
+// launch a kernel on clusters of `cluster` CTAs (grid padded to a multiple)
+template <class... KArgs, class... Args>
+ga_status launch_cluster(void (*k)(KArgs...), uint32_t grid, uint32_t block, uint32_t cluster, cudaStream_t s,
+                         Args... args) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((grid + cluster - 1) / cluster * cluster);
+    cfg.blockDim = dim3(block);
+    cfg.dynamicSmemBytes = 0;
+    cfg.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = cluster;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, k, ((KArgs)args)...) == cudaSuccess ? GA_OK : GA_ECUDA;
+}
+
 }  // namespace
 
 extern "C" {
@@ -343,17 +430,46 @@ ga_status ga_trace_phase(ga_heap_t h, ga_stream_t stream, const uint32_t* sizes,
     if (!h || !sizes || !held || !counts || T == 0 || D > 1) return GA_EINVAL;
     if (block == 0) block = 256;
     DeviceGuard g(h->device);
-    GaPolicy al{ga_dev_heap{h->ddesc, h->dev.base}};
+    const ga_dev_heap dh{h->ddesc, h->dev.base};
+    GaPolicy al{dh};
     cudaStream_t s = (cudaStream_t)stream;
     if (!(flags & GA_TRACE_LOG)) log = nullptr;
+    const uint32_t scope = (flags >> 8) & 0xF;
+    if (!scope_ok(scope, block)) return GA_EINVAL;
+    if (D == 1 ? round > R : (round >= R || phase > 1)) return GA_EINVAL;
     if (D == 1) {
-        if (round > R) return GA_EINVAL;
-        k_churn_round<GaPolicy><<<nblocks(T, block), block, 0, s>>>(al, sizes, R, T, round, held, log, counts, flags);
+        if (scope == 1)
+            k_churn_round<GaBlockPolicy><<<nblocks(T, block), block, 0, s>>>(GaBlockPolicy{dh}, sizes, R, T, round, held, log, counts, flags);
+        else if (scope > 1)
+            return launch_cluster(k_churn_round<GaClusterPolicy>, nblocks(T, block), block, scope, s, GaClusterPolicy{dh},
+                                  sizes, R, T, round, held, log, counts, flags);
+        else k_churn_round<GaPolicy><<<nblocks(T, block), block, 0, s>>>(al, sizes, R, T, round, held, log, counts, flags);
     } else {
-        if (round >= R || phase > 1) return GA_EINVAL;
-        k_phase<GaPolicy><<<nblocks(T, block), block, 0, s>>>(al, sizes, T, round, phase, held, log, counts, flags);
+        if (scope == 1)
+            k_phase<GaBlockPolicy><<<nblocks(T, block), block, 0, s>>>(GaBlockPolicy{dh}, sizes, T, round, phase, held, log, counts, flags);
+        else if (scope > 1)
+            return launch_cluster(k_phase<GaClusterPolicy>, nblocks(T, block), block, scope, s, GaClusterPolicy{dh}, sizes,
+                                  T, round, phase, held, log, counts, flags);
+        else k_phase<GaPolicy><<<nblocks(T, block), block, 0, s>>>(al, sizes, T, round, phase, held, log, counts, flags);
     }
     return launched();
+}
+
+ga_status ga_trace_timed_scope(ga_heap_t h, ga_stream_t stream, const uint32_t* sizes, uint32_t R, uint32_t T, uint32_t D,
+                               uint64_t* counts, uint32_t block, uint32_t scope) {
+    if (scope == 0) return ga_trace_timed(h, stream, sizes, R, T, D, counts, block);
+    if (!h || !sizes || !counts || T == 0 || D > 1) return GA_EINVAL;
+    if (block == 0) block = 256;
+    if (!scope_ok(scope, block)) return GA_EINVAL;
+    DeviceGuard g(h->device);
+    const ga_dev_heap dh{h->ddesc, h->dev.base};
+    cudaStream_t s = (cudaStream_t)stream;
+    if (scope == 1) {
+        k_timed<GaBlockPolicy, 4><<<nblocks(T, block), block, 0, s>>>(GaBlockPolicy{dh}, sizes, R, T, D, counts);
+        return launched();
+    }
+    return launch_cluster(k_timed<GaClusterPolicy, 4>, nblocks(T, block), block, scope, s, GaClusterPolicy{dh}, sizes, R,
+                          T, D, counts);
 }
 
 ga_status ga_trace_timed(ga_heap_t h, ga_stream_t stream, const uint32_t* sizes, uint32_t R, uint32_t T, uint32_t D,

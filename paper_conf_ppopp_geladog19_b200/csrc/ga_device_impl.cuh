@@ -29,6 +29,7 @@
 //     available nodes of order n, every D == 0.
 #pragma once
 #include <cstdint>
+#include <cooperative_groups.h>
 #include "ga.h"
 
 namespace ga {
@@ -254,6 +255,25 @@ static __device__ __forceinline__ uint32_t nth_set(uint64_t x, uint32_t n) {
     return pos;
 }
 
+// OR of v over my group g, for groups that partition the uniform mask m, with
+// every collective on m.  A collective whose mask differs between the lanes
+// executing it (e.g. __reduce_or_sync(g)) compiles to a divergent path
+// (BRA.DIV ... ENDCOLLECTIVE) that runs the groups one after another: on the
+// mixed trace the free path ran with 1 active lane per instruction.  Here the
+// trip count is the largest group's size, uniform over m.
+static __device__ __forceinline__ uint64_t group_or(unsigned m, unsigned g, uint64_t v) {
+    if (__all_sync(m, g == m))                                // one group (warp-uniform calls)
+        return ((uint64_t)__reduce_or_sync(m, (uint32_t)(v >> 32)) << 32) | __reduce_or_sync(m, (uint32_t)v);
+    const uint32_t n = __reduce_max_sync(m, (uint32_t)__popc(g));
+    const uint32_t mine = __popc(g);
+    uint64_t acc = 0;
+    for (uint32_t j = 0; j < n; j++) {
+        const int src = j < mine ? (int)nth_set((uint64_t)g, j) : (int)lane_id();
+        const uint64_t x = __shfl_sync(m, v, src);
+        if (j < mine) acc |= x;
+    }
+    return acc;
+}
 static __device__ __forceinline__ bool is_span(int c) { return c >= kNbin; }
 static __device__ __forceinline__ uint32_t slots_of(int c) { return c < kNbin ? 256u >> c : kChunkPages >> (c - kNbin); }
 // first page of the bin / span holding page p (its slot bitmap and kind live there)
@@ -269,14 +289,19 @@ static __device__ __forceinline__ uint32_t arena_of(const ga_desc* h) { return s
 // (37 MiB) for a class whatever its live set: at full occupancy a 16 B class
 // holds 4.6 MiB live and the reserve dominated fragmentation (7.8x the
 // oracle's on d3).  The tiny classes share arenas so an arena's live set of
-// the class is about a chunk; spans share GA_SPAN_SHARE SMs.
+// the class at full occupancy (2,048 threads per SM) is a little UNDER a whole
+// number of chunks: 7 SMs x 2,048 x 16 B = 56 pages, x 32 B = 112, x 64 B =
+// 224 (7/8 of 1, 2, 4 chunks).  Exactly one chunk's worth (8 SMs at 16 B, 4 at
+// 32 B) spilled into a second chunk whenever a few extra bins were grown
+// (d3 fragmentation 1.46x the oracle's at 16 / 32 B).  Spans share
+// GA_SPAN_SHARE SMs.
 #ifndef GA_SMALL_SHARE
 #define GA_SMALL_SHARE 1
 #endif
 static __device__ __forceinline__ uint32_t class_share(int c) {
     if (c >= kNbin) return GA_SPAN_SHARE;
 #if GA_SMALL_SHARE
-    return c == 0 ? 8 : c <= 2 ? 4 : c == 3 ? 2 : 1;              // 16 B: 8, 32 / 64 B: 4, 128 B: 2
+    return c <= 2 ? 7 : c == 3 ? 2 : 1;                           // 16 / 32 / 64 B: 7, 128 B: 2
 #else
     return 1;
 #endif
@@ -1004,8 +1029,8 @@ static __shared__ uint32_t s_chunk_hint[kNcls];
 // A chunk of arena A with non-full class-c bins, and its non-full page mask:
 // the hint's chunk first, then the (A, c) summary.  Spins until one shows up
 // (the caller holds units, so a free slot exists or is being published).
+static __device__ __noinline__ uint64_t bin_find_chunk_search(const ga_desc* h, uint32_t A, int c, uint64_t* mask_out);
 static __device__ GA_CLAIM_FN uint64_t bin_find_chunk(const ga_desc* h, uint32_t A, int c, uint64_t* mask_out) {
-    GA_DBG_CNT;
 #if GA_HINT_LDCA
     // the hint is only a hint: an L1-cached (possibly stale) read saves an L2
     // round trip; the chunk's owner and non-full word below are read fresh
@@ -1018,6 +1043,11 @@ static __device__ GA_CLAIM_FN uint64_t bin_find_chunk(const ga_desc* h, uint32_t
         uint64_t m = ld_rlx(nonfull_word(h, hp >> kChunkShift, c));
         if (own == A + 1 && m) { s_chunk_hint[c] = hp; *mask_out = m; return hp >> kChunkShift; }
     }
+    return bin_find_chunk_search(h, A, c, mask_out);
+}
+// the (A, c) summary search behind the hint (out of line: rare, and it spins)
+static __device__ __noinline__ uint64_t bin_find_chunk_search(const ga_desc* h, uint32_t A, int c, uint64_t* mask_out) {
+    GA_DBG_CNT;
     HB3 nb = arena_hb(h, A, kAhbNfc + c);
     uint32_t seed = scatter_seed();
     uint32_t ns = 32, spins = 0;
@@ -1048,6 +1078,28 @@ static __device__ GA_CLAIM_FN uint64_t bin_find_chunk(const ga_desc* h, uint32_t
         seed = hash32(seed + 7);
         if ((++spins & 255) == 0) nfc_repair(h, A, c);
     }
+}
+
+// Spans: one candidate per CHUNK, so a chunk's non-full mask names one span
+// and a group needing more slots than one span holds would take one span per
+// iteration (36 warp iterations per call on d3 64 KiB).  Instead the leader
+// takes a whole level-0 word of the (A, c) non-full summary: up to 64 spans
+// with free slots, over which the group's lanes spread by rank.  Returns the
+// summary word index j; *mask_out = its chunk bits (non-zero).  Stale bits
+// are validated by the claim (page kind) and cleaned by the claimer.
+static __device__ __forceinline__ uint64_t span_find_word(const ga_desc* h, uint32_t A, int c, uint64_t* mask_out) {
+    HB3 nb = arena_hb(h, A, kAhbNfc + c);
+    const uint32_t hp = ld_rlx32(&h->hint[A * kNcls + c]);
+    if (hp < h->pages) {
+        const uint64_t j = (uint64_t)hp >> (2 * kChunkShift);
+        const uint64_t m = ld_rlx(&nb.w0[j]);
+        if (m) { *mask_out = m; return j; }
+    }
+    uint64_t m1;
+    const uint64_t ch = bin_find_chunk_search(h, A, c, &m1);             // spins until a span shows up
+    const uint64_t j = ch >> kChunkShift;
+    *mask_out = ld_rlx(&nb.w0[j]) | (1ull << (ch & 63));
+    return j;
 }
 
 // ---------------------------------------------------------------------------
@@ -1362,6 +1414,7 @@ static __device__ __noinline__ uint64_t bin_claim_collective(const ga_desc* h, u
 #endif
             if ((int)lane == L) {
                 if (pre_m) { ch = pre_ch; m = pre_m; pre_m = 0; }                   // loaded beside the semaphore
+                else if (is_span(c)) ch = span_find_word(h, A, c, &m);              // spans: a summary word
                 else ch = bin_find_chunk(h, A, c, &m);
             }
             ch = __shfl_sync(unsat, ch, L);
@@ -1369,12 +1422,18 @@ static __device__ __noinline__ uint64_t bin_claim_collective(const ga_desc* h, u
         }
         const uint32_t q = __popc(unsat & lanemask_lt());
         const uint32_t np = __popcll(m);
-        const uint64_t page = ch * kChunkPages + nth_set(m, (q / per_page + rot + it++) % np);
+        uint64_t page = (ch << kChunkShift) + nth_set(m, (q / per_page + rot + it++) % np);
+        if (is_span(c)) page <<= kChunkShift;                  // spans: summary word -> span head page
         const unsigned pg = __match_any_sync(unsat, page);
         const int pl = __ffs(pg) - 1;
         uint64_t got = 0;
         int wi = 0;
-        if ((int)lane == pl) got = bin_claim_page(h, page, A, c, __popc(pg), &wi, rot >> 8);
+        if ((int)lane == pl) {
+            got = bin_claim_page(h, page, A, c, __popc(pg), &wi, rot >> 8);
+            if (!got && is_span(c))                            // a full or stale span: drop its summary bit
+                hb3_clear_owned(h, arena_hb(h, A, kAhbNfc + c), page >> kChunkShift, A,
+                                nonfull_word(h, page >> kChunkShift, c), 0);
+        }
         got = __shfl_sync(pg, got, pl);
         wi = __shfl_sync(pg, wi, pl);
         const uint32_t pr = __popc(pg & lanemask_lt());
@@ -1638,6 +1697,7 @@ static __device__ __forceinline__ uint64_t malloc_in_arena(const ga_desc* h, uns
             pre_ch = hp >> kChunkShift;
             own = ld_rlx32(&h->chunk_owner[pre_ch]);
             pre_m = ld_rlx(nonfull_word(h, pre_ch, c));
+            if (is_span(c)) own = 0;                              // spans claim over summary words
         }
         r = bsem_decide(sp, old, N, Bp, &w);
         if (r == kBlocked) r = bsem_wait_slow<2048>(sp, N, Bp, ArenaSpin{h, A}, w);
@@ -1646,6 +1706,126 @@ static __device__ __forceinline__ uint64_t malloc_in_arena(const ga_desc* h, uns
     r = __shfl_sync(grp, r, leader);
     return r == kAcquired ? bin_claim_collective(h, grp, A, c, pre_ch, pre_m)
          : is_span(c) ? span_grow_collective(h, grp, A, c) : bin_grow_collective(h, grp, A, c);
+}
+
+#ifndef GA_LOCKSTEP
+#define GA_LOCKSTEP 1            // 1: the bin/span fast path runs every class group of a warp in one instruction stream
+#endif
+// The bin / span fast path with every class group of the warp in ONE
+// instruction stream.  malloc_in_arena runs a group at a time: on a mixed
+// trace a warp holds ~12 class groups, and under independent thread
+// scheduling they issued their own copies of the claim loop one after the
+// other (4.1 active lanes per instruction, ~4,700 warp instructions per
+// warp-call).  Here the control flow is uniform over `bl` (every bin/span
+// lane of the call): leaders issue their Alg. 1 fetch-adds as one
+// instruction, per-group values travel by shuffles from each lane's own group
+// leader, and the claim loop runs while ANY lane of the warp still needs a
+// slot -- so the groups' L2 round trips overlap instead of adding up.  The
+// per-group work is exactly malloc_in_arena's (one wait of N units per group,
+// collective claim by rank over the chunk's non-full pages, one atomicOr per
+// page word); only the schedule differs.  Groups whose wait
+// blocks or says GROW take the per-group path afterwards.
+// A group whose wait did not grant at once: a blocked wait (reservation taken
+// by bsem_decide, re-polled from a fresh load), then the claim or growth.
+// Out of line: rare, and its state would otherwise stay live (and spill)
+// across the lockstep loop.
+static __device__ __noinline__ uint64_t malloc_group_slow(const ga_desc* h, unsigned grp, uint32_t A, int c, int r) {
+    const uint32_t N = __popc(grp), slots = slots_of(c);
+    const uint32_t Bp = slots * ((N + slots - 1) / slots);                         // R-8
+    const int leader = __ffs(grp) - 1;
+    if ((int)lane_id() == leader && r == kBlocked) {
+        uint64_t* sp = sem_ptr(h, A, c);
+        r = bsem_wait_slow<2048>(sp, N, Bp, ArenaSpin{h, A}, ld_rlx(sp));
+    }
+    r = __shfl_sync(grp, r, leader);
+    return r == kAcquired ? bin_claim_collective(h, grp, A, c)
+         : is_span(c) ? span_grow_collective(h, grp, A, c) : bin_grow_collective(h, grp, A, c);
+}
+// held: the group's units were already acquired for it (the block / cluster
+// collective's one wait per class, section 8): no fetch-add here.
+static __device__ __forceinline__ uint64_t malloc_lockstep(const ga_desc* h, unsigned bl, unsigned grp, int c,
+                                                           uint32_t A, bool held = false) {
+    const uint32_t lane = lane_id();
+    const int leader = __ffs(grp) - 1;
+    int r = kAcquired;
+    uint64_t pre_m = 0;
+    uint32_t hp = 0;
+    if ((int)lane == leader) {
+        const uint32_t N = __popc(grp), slots = slots_of(c);
+        const uint32_t Bp = slots * ((N + slots - 1) / slots);                     // R-8
+        uint64_t* sp = sem_ptr(h, A, c);
+        uint64_t w;
+        hp = GA_PREFETCH ? s_chunk_hint[c] : 0xFFFFFFFFu;
+        const uint64_t old = held ? 0 : a_add(sp, dCD(-(int32_t)N, (int32_t)Bp)); // Alg. 1, first fetch-add
+        uint32_t own = 0;
+        if (hp < h->pages) {                                                     // in flight with the fetch-add
+            if (is_span(c)) {                                                    // spans: the hint's summary word
+                own = A + 1;
+                pre_m = ld_rlx(&arena_hb(h, A, kAhbNfc + c).w0[hp >> (2 * kChunkShift)]);
+            } else {
+                own = ld_rlx32(&h->chunk_owner[hp >> kChunkShift]);
+                pre_m = ld_rlx(nonfull_word(h, hp >> kChunkShift, c));
+            }
+        }
+        if (!held) r = bsem_decide(sp, old, N, Bp, &w);
+        if (own != A + 1) pre_m = 0;
+    }
+    r = __shfl_sync(bl, r, leader);
+    const uint32_t per_page = slots_of(c) < 64 ? slots_of(c) : 64;
+    uint32_t wid; asm volatile("mov.u32 %0, %%warpid;" : "=r"(wid));
+    const uint32_t rot = hash32(wid ^ (smid() << 6));
+    uint64_t my = kNull;
+    bool need = r == kAcquired;
+#if GA_COUNT_ITERS
+    if ((int)lane == __ffs(bl) - 1) stat_add(h, kStatRepairNonfull, 1);                // lockstep calls (diagnostic)
+#endif
+    for (uint32_t it = 0;; it++) {
+        const unsigned un = __ballot_sync(bl, need);
+        if (un == 0) break;
+#if GA_COUNT_ITERS
+        if ((int)lane == __ffs(bl) - 1) stat_add(h, kStatRepairSummary, 1);           // warp iterations
+#endif
+        const unsigned g = grp & un;                           // my group's lanes still without a slot
+        const int L = need ? __ffs(g) - 1 : (int)lane;
+        uint64_t ch = 0, m = 0;
+        if (need && (int)lane == L) {
+            if (pre_m) { ch = hp >> (is_span(c) ? 2 * kChunkShift : kChunkShift); m = pre_m; pre_m = 0; }   // loaded beside the semaphore
+            else if (is_span(c)) ch = span_find_word(h, A, c, &m);
+            else ch = bin_find_chunk(h, A, c, &m);
+        }
+        ch = __shfl_sync(bl, ch, L);
+        m = __shfl_sync(bl, m, L);
+        uint64_t key = kNull;
+        uint64_t page = 0;
+        if (need) {
+            const uint32_t q = __popc(g & lanemask_lt());
+            // bins: page of chunk ch; spans: head page of chunk 64 * ch + bit (span_find_word)
+            page = (ch << kChunkShift) + nth_set(m, (q / per_page + rot + it) % (uint32_t)__popcll(m));
+            if (is_span(c)) page <<= kChunkShift;
+            key = (page << 4) | (uint64_t)c;                   // a stale bit can name one page in two classes
+        }
+        const unsigned pg = __match_any_sync(bl, key);
+        const int pl = __ffs(pg) - 1;
+        uint64_t got = 0;
+        int wi = 0;
+        if (need && (int)lane == pl) {
+            got = bin_claim_page(h, page, A, c, __popc(pg), &wi, rot >> 8);
+            if (!got && is_span(c))                            // a full or stale span: drop its summary bit
+                hb3_clear_owned(h, arena_hb(h, A, kAhbNfc + c), page >> kChunkShift, A,
+                                nonfull_word(h, page >> kChunkShift, c), 0);
+        }
+        got = __shfl_sync(bl, got, pl);
+        wi = __shfl_sync(bl, wi, pl);
+        if (need) {
+            const uint32_t pr = __popc(pg & lanemask_lt());
+            if (pr < (uint32_t)__popcll(got)) {
+                my = (page << kPageShift) + ((uint64_t)(wi * 64 + nth_set(got, pr)) << (c + kMinShift));
+                need = false;
+            }
+        }
+    }
+    if (r != kAcquired) my = malloc_group_slow(h, grp, A, c, r);    // per group: blocked wait, growth
+    return my;
 }
 
 // The group-level fallback (R-26: a malloc fails only if no arena
@@ -1723,15 +1903,25 @@ static __device__ __noinline__ uint64_t ga_malloc_off(const ga_desc* h, uint64_t
     if ((int)lane == __ffs(act) - 1) red_rlx(arena_ctr(h, 0), __popc(act));       // n_malloc, per warp
     const int key = size_key(h, n);
     const unsigned grp = __match_any_sync(act, key);
+#if GA_LOCKSTEP
+    const unsigned bl = __match_any_sync(act, (unsigned)(key >= 0 && key < kNcls));   // valid in bin/span lanes
+#endif
     if (key < 0) return kNull;
     uint64_t my;
     if (key < kNcls) {
         const uint32_t A = arena_of(h) / class_share(key);
+#if GA_LOCKSTEP
+        my = malloc_lockstep(h, bl, grp, key, A);
+        // my group's unserved lanes, as a match on the uniform mask bl (see
+        // group_or and active_lanes: no ballot result as a _sync mask)
+        const unsigned rest = __match_any_sync(bl, ((unsigned)key << 1) | (unsigned)(my == kNull));
+#else
         my = malloc_in_arena(h, grp, A, key, true);
-        if (__any_sync(grp, my == kNull)) {
-            const unsigned rest = lanes_where(grp, my == kNull);
-            if ((int)lane == __ffs(grp) - 1) stat_add(h, kStatFallback, 1);
-            if (my == kNull) my = group_fallback(h, rest, A, key);
+        const unsigned rest = lanes_where(grp, my == kNull);
+#endif
+        if (my == kNull) {
+            if ((int)lane == __ffs(rest) - 1) stat_add(h, kStatFallback, 1);
+            my = group_fallback(h, rest, A, key);
         }
         return my;
     }
@@ -1752,7 +1942,10 @@ static __device__ __noinline__ uint64_t ga_malloc_off(const ga_desc* h, uint64_t
 // pair up with __match_any_sync and continue with the parent -- a collective
 // free), then each surviving block runs the merge-on-free protocol; bin slots
 // are grouped per bitmap word (one atomicAnd) and per (arena, class) (one signal).
-static __device__ __noinline__ void ga_free_off(const ga_desc* h, uint64_t off) {
+struct CollState;
+static __device__ __forceinline__ void coll_signal(const ga_desc* h, CollState* R, uint32_t A, int c, uint32_t n);
+template <bool kColl>
+static __device__ __forceinline__ void free_body(const ga_desc* h, uint64_t off, CollState* R) {
     const unsigned act = active_lanes();
     uint32_t k = 0;
     uint64_t p = 0;
@@ -1792,7 +1985,7 @@ static __device__ __noinline__ void ga_free_off(const ga_desc* h, uint64_t off) 
     const int w = (int)(slot >> 6);
     const unsigned g1 = __match_any_sync(bins, (p << 2) | (uint64_t)w);
     const uint64_t bit = 1ull << (slot & 63);
-    const uint64_t mask = ((uint64_t)__reduce_or_sync(g1, (uint32_t)(bit >> 32)) << 32) | __reduce_or_sync(g1, (uint32_t)bit);
+    const uint64_t mask = group_or(bins, g1, bit);
     bool eager = false;
     if ((int)lane_id() == __ffs(g1) - 1) {
         uint64_t* bw = page_bits(h, p);
@@ -1816,10 +2009,172 @@ static __device__ __noinline__ void ga_free_off(const ga_desc* h, uint64_t off) 
     // the units signalled below never precede their slots (no __syncwarp: see
     // active_lanes)
     const unsigned g2 = __match_any_sync(bins, (A << 4) | (uint32_t)c);     // class < 16
-    if ((int)lane_id() == __ffs(g2) - 1) bsem_signal_after_rmw(sem_ptr(h, A, c), __popc(g2));
+    if ((int)lane_id() == __ffs(g2) - 1) {
+        if (kColl) coll_signal(h, R, A, c, __popc(g2));       // block / cluster: one signal per class later
+        else bsem_signal_after_rmw(sem_ptr(h, A, c), __popc(g2));
+    }
     if (eager) {
         fence();                                               // our slots' units are published
         if (!bin_reclaim(h, p, slots_of(c))) mark_candidate(h, p, A);
+    }
+}
+static __device__ __noinline__ void ga_free_off(const ga_desc* h, uint64_t off) { free_body<false>(h, off, nullptr); }
+
+
+// ---------------------------------------------------------------------------
+// 8. block- and cluster-collective entry points.  The paper's
+// collective synchronization primitives work at thread-block scope (Sec.
+// 4.2.2): the threads of a block enter one critical section
+// together, one elected thread performs the synchronization operation for all
+// ("collective acquire": elected acquire + barrier; "collective release":
+// barrier + elected release).  Here EVERY thread of the CTA (block scope) or
+// of the thread-block cluster (cluster scope, CTAs joined through distributed
+// shared memory) calls ga_malloc_block / ga_malloc_cluster together, like
+// __syncthreads():
+//   1. each warp's class groups add their demand to per-class counters in the
+//      collective's shared memory (the root CTA's, through DSMEM for a
+//      cluster);
+//   2. one barrier; then ONE thread per class runs Alg. 1 for the whole
+//      collective's demand of that class -- one semaphore fetch-add for up to
+//      kCollMax threads instead of one per warp group (collective acquire);
+//   3. a second barrier; every warp claims its slots through the lockstep
+//      claim with the units already held (one atomicOr per bitmap word).
+// A wait that says GROW is retracted (signal(0, B'-N)) and the
+// groups of that class run their own waits and growth (the warp path).
+// ga_free_block / ga_free_cluster free through the warp path and add the
+// released units of the collective's own arena to per-class counters; after
+// one barrier the root CTA issues ONE signal per class (collective release).
+// TBuddy sizes (above 64 KiB) take the warp path.  The counters are
+// double-buffered by a parity word, so a malloc needs two barriers and a free
+// one: a class's decider zeroes its counter of the previous call, which every
+// thread finished with before this call's first barrier.  ga_coll_begin
+// zeroes the state once per kernel.
+// ---------------------------------------------------------------------------
+constexpr uint32_t kCollMax = 2048;              // threads of one block- or cluster-collective call
+struct CollState {
+    uint32_t cnt[2][kNcls];       // demand per class, double-buffered by `parity`
+    uint32_t held[kNcls];         // 1: the class's demand was acquired for the collective this call
+    uint32_t sig[kNcls];          // free: units owed to the collective arena's class semaphores
+    uint32_t parity;
+    uint32_t arena;               // arena_of() of the root CTA's SM
+};
+static __device__ __forceinline__ CollState* coll_local() {
+    __shared__ CollState s;                      // one per CTA, only in kernels that use the collective calls
+    return &s;
+}
+template <bool kCluster>
+struct Coll {
+    static __device__ __forceinline__ CollState* root() {
+        if constexpr (kCluster) return cooperative_groups::this_cluster().map_shared_rank(coll_local(), 0u);
+        else return coll_local();
+    }
+    static __device__ __forceinline__ void sync() {
+        if constexpr (kCluster) cooperative_groups::this_cluster().sync();
+        else __syncthreads();
+    }
+    static __device__ __forceinline__ uint32_t rank() {
+        if constexpr (kCluster) return cooperative_groups::this_cluster().block_rank();
+        else return 0;
+    }
+    static __device__ __forceinline__ uint32_t ncta() {
+        if constexpr (kCluster) return cooperative_groups::this_cluster().num_blocks();
+        else return 1;
+    }
+};
+static __device__ __forceinline__ uint32_t cta_tid() { return threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z); }
+static __device__ __forceinline__ uint32_t cta_threads() { return blockDim.x * blockDim.y * blockDim.z; }
+
+static __device__ __forceinline__ void coll_signal(const ga_desc* h, CollState* R, uint32_t A, int c, uint32_t n) {
+    if (A == R->arena / class_share(c)) atomicAdd(&R->sig[c], n);
+    else bsem_signal_after_rmw(sem_ptr(h, A, c), n);
+}
+
+template <bool kCluster>
+static __device__ __noinline__ void coll_begin(const ga_desc* h) {
+    CollState* L = coll_local();
+    const uint32_t t = cta_tid();
+    if (t < 2 * kNcls) (&L->cnt[0][0])[t] = 0;
+    if (t < kNcls) L->sig[t] = 0;
+    if (t == 0) { L->parity = 0; L->arena = arena_of(h); }
+    Coll<kCluster>::sync();
+}
+
+// One thread decides class c for the whole collective: ONE Alg. 1 wait for
+// the collective's demand Nc (B' = slots * ceil(Nc / slots), R-8).  ACQUIRED:
+// every requesting group then claims with its units already held.  GROW is
+// retracted (signal(0, B'-N)) and the groups run their own waits
+// and growth; a blocked wait spins here first (delegating reclamation).
+static __device__ __noinline__ void coll_decide_class(const ga_desc* h, CollState* R, uint32_t par, int c) {
+    R->cnt[par ^ 1][c] = 0;                                          // the previous call's counter
+    const uint32_t Nc = R->cnt[par][c];
+    uint32_t held = 0;
+    if (Nc) {
+        const uint32_t A = R->arena / class_share(c);
+        const uint32_t slots = slots_of(c);
+        const uint32_t Bp = slots * ((Nc + slots - 1) / slots);
+        uint64_t* sp = sem_ptr(h, A, c);
+        uint64_t w = 0;
+        int r = bsem_decide(sp, a_add(sp, dCD(-(int32_t)Nc, (int32_t)Bp)), Nc, Bp, &w);
+        if (r == kBlocked) r = bsem_wait_slow<2048>(sp, Nc, Bp, ArenaSpin{h, A}, w);
+        if (r == kGrow) bsem_signal(sp, 0, Bp - Nc);
+        held = r == kAcquired;
+    }
+    R->held[c] = held;
+}
+
+template <bool kCluster>
+static __device__ __noinline__ uint64_t malloc_coll_off(const ga_desc* h, uint64_t n) {
+    using CC = Coll<kCluster>;
+    CollState* R = CC::root();
+    const unsigned act = active_lanes();
+    const uint32_t lane = lane_id();
+    if ((int)lane == __ffs(act) - 1) red_rlx(arena_ctr(h, 0), __popc(act));       // n_malloc, per warp
+    const int key = size_key(h, n);
+    const bool bin = key >= 0 && key < kNcls;
+    const unsigned grp = __match_any_sync(act, key);
+    const unsigned bl = __match_any_sync(act, (unsigned)bin);                      // valid in bin/span lanes
+    const uint32_t par = R->parity;
+    if (bin && (int)lane == __ffs(grp) - 1) atomicAdd(&R->cnt[par][key], (uint32_t)__popc(grp));
+    CC::sync();                                                                     // demand complete
+    const uint32_t t = cta_tid(), nc = CC::ncta(), me = CC::rank();
+    if (me == 0 && t == 0) R->parity = par ^ 1;
+    if (t * nc + me < (uint32_t)kNcls) coll_decide_class(h, R, par, (int)(t * nc + me));   // class c: CTA c % nc
+    CC::sync();                                                                     // every decision made
+    if (key < 0) return kNull;
+    uint64_t my;
+    if (bin) {
+        const uint32_t A = R->arena / class_share(key);
+        my = malloc_lockstep(h, bl, grp, key, A, R->held[key] != 0);
+        const unsigned rest = __match_any_sync(bl, ((unsigned)key << 1) | (unsigned)(my == kNull));
+        if (my == kNull) {
+            if ((int)lane == __ffs(rest) - 1) stat_add(h, kStatFallback, 1);
+            my = group_fallback(h, rest, A, key);
+        }
+        return my;
+    }
+    const int o = key - kNcls;                                                      // TBuddy: the warp path
+    my = tree_malloc_group(h, grp, o);
+    if (my == kNull) {
+        int64_t x = tree_alloc_one_retry(h, o, false);
+        if (x >= 0) {
+            uint64_t pgt = (uint64_t)x << o;
+            st_rlx32(&h->kind[pgt], kKindTree | (uint32_t)o);
+            my = pgt << kPageShift;
+        } else stat_add(h, kStatFail, 1);
+    }
+    return my;
+}
+
+template <bool kCluster>
+static __device__ __noinline__ void free_coll_off(const ga_desc* h, uint64_t off) {
+    using CC = Coll<kCluster>;
+    CollState* R = CC::root();
+    free_body<true>(h, off, R);
+    CC::sync();                                                                     // every unit counted
+    const uint32_t t = cta_tid();
+    if (CC::rank() == 0 && t < kNcls) {
+        const uint32_t v = atomicExch(&R->sig[t], 0u);
+        if (v) bsem_signal_after_rmw(sem_ptr(h, R->arena / class_share((int)t), (int)t), v);
     }
 }
 

@@ -7,9 +7,9 @@ from dataclasses import dataclass, field
 import numpy as np
 import torch
 
-from . import (GA_TRACE_LOG, GA_TRACE_TAG, ga_cuda_trace_phase, ga_cuda_trace_timed, ga_heap_create,
+from . import (GA_TRACE_LOG, GA_TRACE_SCOPE, GA_TRACE_TAG, ga_cuda_trace_phase, ga_cuda_trace_timed, ga_heap_create,
                ga_heap_destroy, ga_heap_quiesce, ga_heap_reset, ga_heap_snapshot, ga_heap_info,
-               ga_reserved_pages, ga_stats, ga_trace_phase, ga_trace_timed, ga_trace_timed_host)
+               ga_reserved_pages, ga_stats, ga_trace_phase, ga_trace_timed, ga_trace_timed_host, ga_trace_timed_scope)
 
 LOG_DTYPE = np.dtype([("off", "<u8"), ("size", "<u4"), ("meta", "<u4")])
 PAGE = 4096
@@ -77,9 +77,10 @@ def _counts(t: torch.Tensor) -> dict:
 
 
 def run_correctness(heap: GpuHeap | None, sizes: np.ndarray, D: int, log: bool = True, tag: bool = True,
-                    reserved: bool = True, block: int = 256) -> TraceRun:
+                    reserved: bool = True, block: int = 256, scope: int = 0) -> TraceRun:
     """Correctness mode: one kernel per phase, log + lifetime tags; reserved pages
-    read at each phase boundary (after a round's mallocs).  heap=None runs CUDA malloc."""
+    read at each phase boundary (after a round's mallocs).  heap=None runs CUDA malloc.
+    scope: 0 warp calls, 1 block-collective, 2..8 cluster-collective (GA_TRACE_SCOPE)."""
     dev = torch.device("cuda", heap.device if heap else torch.cuda.current_device())
     R, T = sizes.shape
     st = heap.stream if heap else torch.cuda.current_stream()
@@ -91,7 +92,7 @@ def run_correctness(heap: GpuHeap | None, sizes: np.ndarray, D: int, log: bool =
     counts = torch.zeros(8, dtype=torch.int64, device=dev)
     rounds = R + 1 if D == 1 else R
     d_log = torch.zeros(2 * rounds * T * 2, dtype=torch.int64, device=dev) if (log and heap) else None
-    flags = (GA_TRACE_LOG if d_log is not None else 0) | (GA_TRACE_TAG if tag else 0)
+    flags = (GA_TRACE_LOG if d_log is not None else 0) | (GA_TRACE_TAG if tag else 0) | GA_TRACE_SCOPE(scope)
     run = TraceRun({})
     lp = d_log.data_ptr() if d_log is not None else 0
     for r in range(rounds):
@@ -127,10 +128,13 @@ def run_correctness(heap: GpuHeap | None, sizes: np.ndarray, D: int, log: bool =
 
 
 def run_timed(heap: GpuHeap | None, d_sizes: torch.Tensor, R: int, T: int, D: int,
-              counts: torch.Tensor, block: int = 256, stream=None):
-    """Timing mode: one kernel, allocator calls only (heap=None: CUDA malloc)."""
+              counts: torch.Tensor, block: int = 256, stream=None, scope: int = 0):
+    """Timing mode: one kernel, allocator calls only (heap=None: CUDA malloc).
+    scope: 0 warp calls, 1 block-collective, 2..8 cluster-collective."""
     s = _stream(stream)
-    if heap:
+    if heap and scope:
+        ga_trace_timed_scope(heap.h, s, d_sizes.data_ptr(), R, T, D, counts.data_ptr(), block, scope)
+    elif heap:
         ga_trace_timed(heap.h, s, d_sizes.data_ptr(), R, T, D, counts.data_ptr(), block)
     else:
         ga_cuda_trace_timed(s, d_sizes.data_ptr(), R, T, D, counts.data_ptr(), block)

@@ -56,7 +56,7 @@ def time_phase(run_malloc, run_free, reps: int = 2):
     return best
 
 
-def one_size(s: int, cuda: bool, all_blocks: bool) -> dict:
+def one_size(s: int, cuda: bool, all_blocks: bool, reps: int = 2) -> dict:
     import torch
     import paper_conf_ppopp_geladog19_b200 as ga
     from paper_conf_ppopp_geladog19_b200.runner import GpuHeap
@@ -90,7 +90,7 @@ def one_size(s: int, cuda: bool, all_blocks: bool) -> dict:
                 ga.ga_trace_phase(heap.h, st, d.data_ptr(), 1, T, 0, 0, 1, held.data_ptr(), 0, cnt.data_ptr(), 0, blk)
                 heap.reset()
 
-        t = time_phase(mal, fre)
+        t = time_phase(mal, fre, reps)
         res["per_block"][str(blk)] = {"seconds": t, "allocs_per_s": T / t, "failed": max(fails)}
     v = list(res["per_block"].values())
     res["allocs_per_s_block256"] = res["per_block"].get("256", v[0])["allocs_per_s"]
@@ -108,9 +108,10 @@ def main():
     ap.add_argument("--one", type=int, default=0, help="internal: one size in this process")
     ap.add_argument("--cuda", action="store_true", help="internal: CUDA malloc for --one")
     ap.add_argument("--sizes", default=None)
+    ap.add_argument("--reps", type=int, default=2, help="timed malloc phases per block size (best kept)")
     a = ap.parse_args()
     if a.one:
-        print(json.dumps(one_size(a.one, a.cuda, a.all_blocks)))
+        print(json.dumps(one_size(a.one, a.cuda, a.all_blocks, a.reps)))
         return 0
     import oracle
     oracle.build()
@@ -120,7 +121,7 @@ def main():
         row = {"size": s}
         for who in ("ours", "cuda"):
             cmd = [sys.executable, __file__, "--one", str(s)] + (["--cuda"] if who == "cuda" else []) + \
-                  (["--all-blocks"] if a.all_blocks else [])
+                  (["--all-blocks"] if a.all_blocks else []) + ["--reps", str(a.reps)]
             r = subprocess.run(cmd, capture_output=True, text=True, timeout=1200)
             lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
             row[who] = json.loads(lines[-1]) if lines else {"error": (r.stderr or "")[-400:]}

@@ -19,6 +19,8 @@ ap.add_argument("--cuda", action="store_true")
 ap.add_argument("--kmin", type=int, default=3)
 ap.add_argument("--kmax", type=int, default=15)
 ap.add_argument("--threads", type=int, default=0, help="fewer threads than the full grid (sanitizer runs)")
+ap.add_argument("--stats", action="store_true", help="heap stats after every rep")
+ap.add_argument("--scope", type=int, default=0, help="0 warp calls, 1 block-collective, 2..8 cluster-collective")
 ap.add_argument("--warm", action="store_true", help="no heap reset between reps")
 ap.add_argument("--level", default="pressure", help="d4 pressure level (fit / pressure / exhaust / overcommit)")
 a = ap.parse_args()
@@ -42,10 +44,14 @@ for i in range(a.reps):
         heap.reset()                                   # cold heap per rep, as bench.py times it
     s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     s.record()
-    run_timed(heap, d, t.R, t.T, t.D, c)
+    run_timed(heap, d, t.R, t.T, t.D, c, scope=a.scope)
     e.record()
     e.synchronize()
     print(f"rep {i}: {s.elapsed_time(e):.2f} ms, counts {c.cpu().numpy()[:4]}", flush=True)
+    if a.stats and heap is not None:
+        st = heap.stats()
+        print("  ", {k: st[k] for k in ("peak_reserved_bytes", "n_bin_grow", "n_chunk_grow", "n_bin_reclaim", "n_fallback",
+                                      "n_waiter_reclaim", "n_fail")}, flush=True)
 if heap is not None:
     st = heap.stats()
     print("stats", {k: st[k] for k in ("n_repair_nonfull", "n_repair_summary", "n_fallback", "n_fail")}, flush=True)
