@@ -68,7 +68,7 @@ def test_d3_uniform_collective(scope, size):
     """Warp-uniform sizes, every block live at once: one semaphore operation
     per class per CTA / cluster; counts equal the oracle's."""
     T = 16384 + 77                                   # ragged last block
-    heap_bytes = 1 << 30 if size >= 65536 else 256 << 20
+    heap_bytes = 2 << 30 if size >= 65536 else 256 << 20
     sizes = np.full((3, T), size, dtype=np.uint32)
     ref = oracle.run_trace(sizes, heap_bytes, 0)
     heap = GpuHeap(heap_bytes)
