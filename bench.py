@@ -39,6 +39,14 @@ L2_FLUSH_BYTES = 512 << 20
 
 
 # ----------------------------------------------------------------------------- helpers
+_T0 = time.time()
+
+
+def _progress(what: str):
+    """Elapsed wall time of each bench leg on stderr (the JSON line stays on stdout)."""
+    print(f"[bench] {time.time() - _T0:7.1f} s  {what}", file=sys.stderr, flush=True)
+
+
 def algorithmic_atomics(sizes: np.ndarray, group: int = 32) -> int:
     """Minimum L2 atomics the method must issue for one pass of a D=1 trace with
     every call succeeding: per warp-round and size class,
@@ -251,6 +259,7 @@ def d3_sweep(ga, heap, stream, dev, T, args, sizes=(16, 32, 64, 128, 256, 512, 1
         ref = oracle.run_trace(one, heap.heap_bytes, 0, want_ok=False).stats
         fg = run.peak_reserved_bytes / run.peak_live_bytes
         fo = ref["peak_reserved_bytes"] / ref["peak_live_bytes"]
+        _progress(f"d3 {sz} B")
         res[str(sz)] = {"Gcalls_s": ours / 1e9, "cuda_Mcalls_s": cuda / 1e6, "x_cuda": ours / cuda,
                         "failed": fails + int(c[1]) + run.counts["n_fail"],
                         "frag": {"gpu": round(fg, 4), "oracle": round(fo, 4), "ratio": round(fg / fo, 4)}}
@@ -305,6 +314,7 @@ def d4_levels(ga, stream, dev, args, flush, levels=("fit", "exhaust", "overcommi
                    "reclaims": {"bins": int(st["n_bin_reclaim"]), "by_waiters": int(st["n_waiter_reclaim"])}}
         heap.close()
         del d
+        _progress(f"d4 level {lv}")
     return res
 
 
@@ -548,10 +558,15 @@ class GpuArm:
         cpu.pop("stats")
         cpu.pop("seconds")
         out["cpu_baseline"] = cpu
+        _progress("cuda_malloc + fragmentation + cpu_baseline")
         out["d4_levels"] = d4_levels(ga, stream, dev, args, self.flush)
+        _progress("d4_levels")
         out["d3"] = d3_sweep(ga, heap, stream, dev, t.T, args)
+        _progress("d3")
         out["d2"] = d2_bsem(ga, stream, dev)
+        _progress("d2")
         out["cpu_baseline_all_cores"] = oracle_leg_parallel(t)
+        _progress("cpu_baseline_all_cores")
 
 
 def l2_peak(ga, torch, dev, stream):

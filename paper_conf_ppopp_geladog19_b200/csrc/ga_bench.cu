@@ -387,10 +387,13 @@ __global__ void k_bsem_init(uint32_t n_sems, uint64_t* sems, uint32_t variant) {
 }
 
 // resident 256-thread blocks per SM the timed kernel is compiled for (register
-// budget 65536 / (256 * minB)); GA_TIMED_OCC=1..6 or 8 selects.  Default 4 (64
-// registers): measured fastest on d4 (8 forces 32 registers and spills).
+// budget 65536 / (256 * minB)); GA_TIMED_OCC=1..6 or 8 selects.  Default 3 (80
+// registers).  Round-2 sweep (median ms, cold heap): d4
+// 5.2 / 5.7 / 6.5 / 18.6 at 2 / 3 / 4 / 8 blocks per SM -- the allocator's
+// hot loop spills 8 / 168 / 224 / 388 B at those budgets -- while
+// warp-uniform d3 256 B takes 1.15 / 0.95 / 0.85 ms.  3 is the compromise.
 inline int occupancy_target() {
-    static int v = [] { const char* e = getenv("GA_TIMED_OCC"); int x = e ? atoi(e) : 4; return (x >= 1 && x <= 8 && x != 7) ? x : 4; }();
+    static int v = [] { const char* e = getenv("GA_TIMED_OCC"); int x = e ? atoi(e) : 3; return (x >= 1 && x <= 8 && x != 7) ? x : 3; }();
     return v;
 }
 inline uint32_t nblocks(uint32_t T, uint32_t block) { return (T + block - 1) / block; }

@@ -1080,6 +1080,30 @@ static __device__ __noinline__ uint64_t bin_find_chunk_search(const ga_desc* h, 
     }
 }
 
+#ifndef GA_SPREAD
+#define GA_SPREAD 1              // 1: lockstep retries pick their chunk from the hint's summary word by warp rotation
+#endif
+// A retry's chunk: every warp of an SM starts at the same hinted chunk, and a
+// class with few slots per page (2 KiB: 2) fills it long before the warps are
+// served (6-7 warp iterations per call on d3 1-2 KiB).  A retry instead takes
+// the summary word holding the hinted chunk (up to 64 of arena A's chunks with
+// non-full class-c pages) and picks one by the warp's rotation, so the warps
+// of an arena spread over its chunks.  Falls back to bin_find_chunk.
+static __device__ __forceinline__ uint64_t bin_spread_chunk(const ga_desc* h, uint32_t A, int c, uint32_t sel,
+                                                            uint64_t* mask_out) {
+    const uint32_t hp = s_chunk_hint[c];
+    if (hp < h->pages) {
+        const uint64_t w = ld_rlx(&arena_hb(h, A, kAhbNfc + c).w0[hp >> (2 * kChunkShift)]);
+        if (w) {
+            const uint64_t ch = ((uint64_t)(hp >> (2 * kChunkShift)) << kChunkShift) + nth_set(w, sel % (uint32_t)__popcll(w));
+            const uint32_t own = ld_rlx32(&h->chunk_owner[ch]);
+            const uint64_t m = ld_rlx(nonfull_word(h, ch, c));
+            if (own == A + 1 && m) { *mask_out = m; return ch; }
+        }
+    }
+    return bin_find_chunk(h, A, c, mask_out);
+}
+
 // Spans: one candidate per CHUNK, so a chunk's non-full mask names one span
 // and a group needing more slots than one span holds would take one span per
 // iteration (36 warp iterations per call on d3 64 KiB).  Instead the leader
@@ -1804,6 +1828,7 @@ static __device__ __forceinline__ uint64_t malloc_lockstep(const ga_desc* h, uns
         if (need && (int)lane == L) {
             if (pre_m) { ch = hp >> (is_span(c) ? 2 * kChunkShift : kChunkShift); m = pre_m; pre_m = 0; }   // loaded beside the semaphore
             else if (is_span(c)) ch = span_find_word(h, A, c, &m);
+            else if (GA_SPREAD && it > 0) ch = bin_spread_chunk(h, A, c, rot + it, &m);
             else ch = bin_find_chunk(h, A, c, &m);
         }
         ch = __shfl_sync(bl, ch, L);

@@ -41,6 +41,7 @@ def main():
     ap.add_argument("--all-blocks", action="store_true")
     ap.add_argument("--B", type=int, default=512)
     ap.add_argument("--out", default=None)
+    ap.add_argument("--reps", type=int, default=3, help="timed runs per point (best kept)")
     a = ap.parse_args()
     import torch
     import paper_conf_ppopp_geladog19_b200 as ga
@@ -59,7 +60,7 @@ def main():
                 cfg = ga.BsemCfg(variant=v, k=1, B=a.B, n_sems=1, iters=1, acquire_only=1, grid=grid, block=blk,
                                  seed=0)
                 best, ok, over = None, True, 1.0
-                for rep in range(3):
+                for rep in range(a.reps):
                     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                     e0.record()
                     ga.ga_bsem_bench(st, cfg, sems.data_ptr(), out.data_ptr())
