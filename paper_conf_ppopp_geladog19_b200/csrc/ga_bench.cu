@@ -467,10 +467,20 @@ ga_status ga_trace_timed_scope(ga_heap_t h, ga_stream_t stream, const uint32_t* 
     DeviceGuard g(h->device);
     const ga_dev_heap dh{h->ddesc, h->dev.base};
     cudaStream_t s = (cudaStream_t)stream;
+    // the same register budget as the warp path's timed kernel (2, 3 or 4 blocks per SM)
+    const int occ = occupancy_target() <= 2 ? 2 : occupancy_target() == 3 ? 3 : 4;
     if (scope == 1) {
-        k_timed<GaBlockPolicy, 4><<<nblocks(T, block), block, 0, s>>>(GaBlockPolicy{dh}, sizes, R, T, D, counts);
+        if (occ == 2) k_timed<GaBlockPolicy, 2><<<nblocks(T, block), block, 0, s>>>(GaBlockPolicy{dh}, sizes, R, T, D, counts);
+        else if (occ == 3) k_timed<GaBlockPolicy, 3><<<nblocks(T, block), block, 0, s>>>(GaBlockPolicy{dh}, sizes, R, T, D, counts);
+        else k_timed<GaBlockPolicy, 4><<<nblocks(T, block), block, 0, s>>>(GaBlockPolicy{dh}, sizes, R, T, D, counts);
         return launched();
     }
+    if (occ == 2)
+        return launch_cluster(k_timed<GaClusterPolicy, 2>, nblocks(T, block), block, scope, s, GaClusterPolicy{dh}, sizes,
+                              R, T, D, counts);
+    if (occ == 3)
+        return launch_cluster(k_timed<GaClusterPolicy, 3>, nblocks(T, block), block, scope, s, GaClusterPolicy{dh}, sizes,
+                              R, T, D, counts);
     return launch_cluster(k_timed<GaClusterPolicy, 4>, nblocks(T, block), block, scope, s, GaClusterPolicy{dh}, sizes, R,
                           T, D, counts);
 }

@@ -1769,6 +1769,22 @@ static __device__ __forceinline__ uint64_t malloc_in_arena(const ga_desc* h, uns
 // collective claim by rank over the chunk's non-full pages, one atomicOr per
 // page word); only the schedule differs.  Groups whose wait
 // blocks or says GROW take the per-group path afterwards.
+#ifndef GA_FIND_NOINL
+#define GA_FIND_NOINL 0          // 1: the lockstep loop's chunk search out of line (smaller loop code)
+#endif
+#if GA_FIND_NOINL
+#define GA_FIND_FN __noinline__
+#else
+#define GA_FIND_FN __forceinline__
+#endif
+// The chunk (bins) or summary word (spans) a lockstep iteration claims from,
+// when nothing was loaded beside the semaphore.
+static __device__ GA_FIND_FN uint64_t lockstep_find(const ga_desc* h, uint32_t A, int c, uint32_t it, uint32_t rot,
+                                                     uint64_t* m) {
+    if (is_span(c)) return span_find_word(h, A, c, m);
+    if (GA_SPREAD && it > 0) return bin_spread_chunk(h, A, c, rot + it, m);
+    return bin_find_chunk(h, A, c, m);
+}
 // A group whose wait did not grant at once: a blocked wait (reservation taken
 // by bsem_decide, re-polled from a fresh load), then the claim or growth.
 // Out of line: rare, and its state would otherwise stay live (and spill)
@@ -1833,9 +1849,7 @@ static __device__ __forceinline__ uint64_t malloc_lockstep(const ga_desc* h, uns
         uint64_t ch = 0, m = 0;
         if (need && (int)lane == L) {
             if (pre_m) { ch = hp >> (is_span(c) ? 2 * kChunkShift : kChunkShift); m = pre_m; pre_m = 0; }   // loaded beside the semaphore
-            else if (is_span(c)) ch = span_find_word(h, A, c, &m);
-            else if (GA_SPREAD && it > 0) ch = bin_spread_chunk(h, A, c, rot + it, &m);
-            else ch = bin_find_chunk(h, A, c, &m);
+            else ch = lockstep_find(h, A, c, it, rot, &m);
         }
         ch = __shfl_sync(bl, ch, L);
         m = __shfl_sync(bl, m, L);

@@ -8,7 +8,7 @@ cd "$(dirname "$0")/.."
 LIB=${LIB:-paper_conf_ppopp_geladog19_b200/libga.so}
 [ -s gpurun_out/bench_full.json ] && grep '^{' gpurun_out/bench_full.json | tail -1 > profiles/r02_bench.json
 [ -s gpurun_out/launches_bench.csv ] && cp gpurun_out/launches_bench.csv profiles/r02_launches_bench.csv
-tmp=$(mktemp -d); (cd $tmp && cuobjdump -xelf all "$OLDPWD/$LIB" > /dev/null)
+tmp=$(mktemp -d); LIBA=$(readlink -f "$LIB"); (cd $tmp && cuobjdump -xelf all "$LIBA" > /dev/null)
 OCC=${OCC:-3}
 for w in d4 d3_16; do
   [ -s gpurun_out/${w}_timed.ncu-rep ] || continue
