@@ -108,6 +108,7 @@ enum { kStatBinGrow = 0, kStatChunkGrow, kStatBinReclaim, kStatChunkReclaim, kSt
 // the stats block), and the per-arena call counters (ga_stats_t)
 constexpr int kStatReserved = 8, kStatPeakReserved = 12, kStatWords = 16;
 constexpr int kStatWaiterReclaim = 9;           // bins reclaimed by threads blocked in a wait
+constexpr int kStatDrainLock = 10, kStatDrainGen = 11;   // reclaim_all: one drain at a time, and its generation
 constexpr int kActrStride = 8;                  // u64 words per arena: [0] mallocs, [1] frees
 
 static __device__ __forceinline__ uint32_t lane_id() { uint32_t r; asm volatile("mov.u32 %0, %%laneid;" : "=r"(r)); return r; }
@@ -1265,7 +1266,33 @@ static __device__ __noinline__ void reclaim_arenas(const ga_desc* h, uint32_t A0
             if (top[i]) reclaim_arena(h, base + i * step, -1, 0);
     }
 }
-static __device__ __noinline__ void reclaim_all(const ga_desc* h) { reclaim_arenas(h, 0, 1); }
+// Drain every arena's reclaim candidates (failing mallocs, exhausted chunk
+// supply).  One drain runs at a time; a caller that finds one running waits
+// until a drain that STARTED after its arrival has completed (two completed
+// drains past its arrival generation: drains are serialised, so the second
+// began after it arrived and saw every candidate it could have seen), then
+// returns without a scan of its own.  At exhaustion tens of thousands of
+// failing lanes each swept all 148 arenas (a 13 s step at block scope, d3
+// 64 KiB); now they share sweeps.  Same guarantee for every caller: all
+// candidates present at its arrival have been reclaimed or found in use.
+static __device__ __noinline__ void reclaim_all(const ga_desc* h) {
+    uint64_t* lock = &h->stats[kStatDrainLock];
+    uint64_t* gen = &h->stats[kStatDrainGen];
+    const uint64_t g0 = ld_rlx(gen);
+    uint32_t ns = 256;
+    for (;;) {
+        if (ld_rlx(lock) == 0 && a_cas(lock, 0ull, 1ull) == 0ull) {
+            fence();
+            reclaim_arenas(h, 0, 1);
+            fence();
+            a_add(gen, 1);
+            a_exch(lock, 0ull);
+            return;
+        }
+        if (ld_rlx(gen) >= g0 + 2) { fence(); return; }
+        __nanosleep(ns); if (ns < 4096) ns <<= 1;
+    }
+}
 
 // Per-lane TBuddy allocation with the no-false-starvation retry: the optimistic
 // order semaphores can send a lane up the tree while another lane's split is
