@@ -80,6 +80,9 @@ constexpr int kMaxLevels = 48;
 #ifndef GA_TREE_SPIN_CAP
 #define GA_TREE_SPIN_CAP 256     // max __nanosleep backoff (ns) of a blocked TBuddy wait
 #endif
+#ifndef GA_LAZY_CLEAR
+#define GA_LAZY_CLEAR 0          // 1: a claim that fills a page leaves its non-full bit; the next claimer to find it full clears it
+#endif
 #ifndef GA_INL_CLAIM
 #define GA_INL_CLAIM 1           // 1: inline the hint lookup and page claim into the collective claim
 #endif
@@ -904,7 +907,7 @@ static __device__ GA_CLAIM_FN uint64_t bin_claim_page(const ga_desc* h, uint64_t
                     undo_claim(h, p, i, got, k2);
                     return 0;
                 }
-                if (((old | m) | ~vm) == ~0ull) {                  // this word is full now
+                if (!GA_LAZY_CLEAR && ((old | m) | ~vm) == ~0ull) {   // this word is full now
                     ld_bitmap(bw, w);
                     if (page_full(w, c)) nonfull_clear_if_full(h, p, c, A);
                 }

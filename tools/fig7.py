@@ -109,6 +109,7 @@ def main():
     ap.add_argument("--cuda", action="store_true", help="internal: CUDA malloc for --one")
     ap.add_argument("--sizes", default=None)
     ap.add_argument("--reps", type=int, default=2, help="timed malloc phases per block size (best kept)")
+    ap.add_argument("--run-timeout", type=int, default=1200, help="seconds per (size, allocator) subprocess")
     a = ap.parse_args()
     if a.one:
         print(json.dumps(one_size(a.one, a.cuda, a.all_blocks, a.reps)))
@@ -122,9 +123,12 @@ def main():
         for who in ("ours", "cuda"):
             cmd = [sys.executable, __file__, "--one", str(s)] + (["--cuda"] if who == "cuda" else []) + \
                   (["--all-blocks"] if a.all_blocks else []) + ["--reps", str(a.reps)]
-            r = subprocess.run(cmd, capture_output=True, text=True, timeout=1200)
-            lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
-            row[who] = json.loads(lines[-1]) if lines else {"error": (r.stderr or "")[-400:]}
+            try:
+                r = subprocess.run(cmd, capture_output=True, text=True, timeout=a.run_timeout)
+                lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+                row[who] = json.loads(lines[-1]) if lines else {"error": (r.stderr or "")[-400:]}
+            except subprocess.TimeoutExpired:
+                row[who] = {"error": f"timed out after {a.run_timeout} s"}
         T, pool = pool_of(s) // s, pool_of(s)
         ref = oracle.run_trace(np.full((1, T), s, dtype=np.uint32), pool, 0, want_ok=False).stats
         row["oracle_failed"] = ref["n_malloc_fail"]
