@@ -80,6 +80,9 @@ constexpr int kMaxLevels = 48;
 #ifndef GA_TREE_SPIN_CAP
 #define GA_TREE_SPIN_CAP 256     // max __nanosleep backoff (ns) of a blocked TBuddy wait
 #endif
+#ifndef GA_DEFER_RECHECK
+#define GA_DEFER_RECHECK 0       // 1: the lockstep claim validates its slots' page kinds once after the loop, not per iteration
+#endif
 #ifndef GA_LAZY_CLEAR
 #define GA_LAZY_CLEAR 0          // 1: a claim that fills a page leaves its non-full bit; the next claimer to find it full clears it
 #endif
@@ -875,7 +878,7 @@ static __device__ __noinline__ void undo_claim(const ga_desc* h, uint64_t p, int
 // words (scattered search).  Loops stay rolled: this is the hottest
 // code of the allocator and instruction-fetch stalls dominate.
 static __device__ GA_CLAIM_FN uint64_t bin_claim_page(const ga_desc* h, uint64_t p, uint32_t A, int c, int need, int* wi,
-                                                       uint32_t rot) {
+                                                       uint32_t rot, bool recheck = true) {
     uint64_t* bw = page_bits(h, p);
     uint64_t w[4];
     const uint32_t k0 = ld_rlx32(&h->kind[p]);
@@ -900,7 +903,7 @@ static __device__ GA_CLAIM_FN uint64_t bin_claim_page(const ga_desc* h, uint64_t
             uint64_t old = a_or(&bw[i], m);
             uint64_t got = m & ~old;
             if (got) {
-                if (const uint32_t k2 = ld_rlx32(&h->kind[p]); k2 != kind_bin(A, c)) {
+                if (const uint32_t k2 = recheck ? ld_rlx32(&h->kind[p]) : kind_bin(A, c); k2 != kind_bin(A, c)) {
                     // recycled page: undo, then re-publish it for its real
                     // owner (as bin_reclaim's ABA path does): a claimer of
                     // (A', c') may have seen our bits and dropped the page
@@ -1865,6 +1868,7 @@ static __device__ __forceinline__ uint64_t malloc_lockstep(const ga_desc* h, uns
     const uint32_t rot = hash32(wid ^ (smid() << 6));
     uint64_t my = kNull;
     bool need = r == kAcquired;
+    bool checked = false;                                      // GA_DEFER_RECHECK: my slot's incarnation validated
 #if GA_COUNT_ITERS
     if ((int)lane == __ffs(bl) - 1) stat_add(h, kStatRepairNonfull, 1);                // lockstep calls (diagnostic)
 #endif
@@ -1901,7 +1905,7 @@ static __device__ __forceinline__ uint64_t malloc_lockstep(const ga_desc* h, uns
         uint64_t got = 0;
         int wi = 0;
         if (need && (int)lane == pl) {
-            got = bin_claim_page(h, page, A, c, __popc(pg), &wi, rot >> 8);
+            got = bin_claim_page(h, page, A, c, __popc(pg), &wi, rot >> 8, !GA_DEFER_RECHECK);
             if (!got && is_span(c))                            // a full or stale span: drop its summary bit
                 hb3_clear_owned(h, arena_hb(h, A, kAhbNfc + c), page >> kChunkShift, A,
                                 nonfull_word(h, page >> kChunkShift, c), 0);
@@ -1915,6 +1919,35 @@ static __device__ __forceinline__ uint64_t malloc_lockstep(const ga_desc* h, uns
                 need = false;
             }
         }
+#if GA_DEFER_RECHECK
+        if (__ballot_sync(bl, need) == 0) {
+            // Every lane holds a slot: validate them all at once (one parallel
+            // round trip instead of one per iteration).  A slot taken in a page
+            // recycled between the claimer's kind read and its atomicOr (ABA)
+            // belongs to another incarnation; while we hold the bit that
+            // incarnation cannot be reclaimed, so the kind read now decides
+            // (as the immediate recheck did): give the slot back, re-publish
+            // the page for its owner, and claim again.
+            bool bad = false;
+            if (my != kNull && !checked) {
+                const uint64_t pg0 = bin_head(my >> kPageShift, c);
+                const uint32_t k2 = ld_rlx32(&h->kind[pg0]);
+                if (k2 != kind_bin(A, c)) {
+                    const uint32_t slot = (uint32_t)((my - (pg0 << kPageShift)) >> (c + kMinShift));
+                    a_and(&page_bits(h, pg0)[slot >> 6], ~(1ull << (slot & 63)));
+                    if ((k2 & 0xC0000000u) == kKindBin) {
+                        nonfull_set(h, pg0, (int)(k2 & 0xFF), (k2 >> 8) & 0xFFFFu);
+                        mark_candidate(h, pg0, (k2 >> 8) & 0xFFFFu);
+                    }
+                    my = kNull;
+                    need = true;
+                    bad = true;
+                }
+            }
+            checked = !bad && my != kNull;
+            if (!__any_sync(bl, bad)) break;
+        }
+#endif
     }
     if (r != kAcquired) my = malloc_group_slow(h, grp, A, c, r);    // per group: blocked wait, growth
     return my;
