@@ -100,8 +100,8 @@ __device__ __forceinline__ void flush_counts(uint64_t* counts, uint32_t nm, uint
 
 // D == 1 correctness round r in [0, R]: free the held block, then malloc (r < R).
 // Collective policies keep threads t >= T in every call (free NULL, malloc 0).
-template <class P>
-__global__ void __launch_bounds__(256) k_churn_round(P al, const uint32_t* sizes, uint32_t R, uint32_t T, uint32_t r,
+template <class P, int MAXB = 256>
+__global__ void __launch_bounds__(MAXB) k_churn_round(P al, const uint32_t* sizes, uint32_t R, uint32_t T, uint32_t r,
                                                      uint64_t* held, ga_log_rec* log, uint64_t* counts, uint32_t flags) {
     uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
     if (!P::kColl && t >= T) return;
@@ -144,8 +144,8 @@ __global__ void __launch_bounds__(256) k_churn_round(P al, const uint32_t* sizes
 }
 
 // D == 0 correctness: phase 0 mallocs every round-r block, phase 1 frees them
-template <class P>
-__global__ void __launch_bounds__(256) k_phase(P al, const uint32_t* sizes, uint32_t T, uint32_t r, uint32_t phase,
+template <class P, int MAXB = 256>
+__global__ void __launch_bounds__(MAXB) k_phase(P al, const uint32_t* sizes, uint32_t T, uint32_t r, uint32_t phase,
                                                uint64_t* held, ga_log_rec* log, uint64_t* counts, uint32_t flags) {
     uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
     if (!P::kColl && t >= T) return;
@@ -423,6 +423,28 @@ ga_status launch_cluster(void (*k)(KArgs...), uint32_t grid, uint32_t block, uin
     return cudaLaunchKernelEx(&cfg, k, ((KArgs)args)...) == cudaSuccess ? GA_OK : GA_ECUDA;
 }
 
+template <int MAXB>
+ga_status trace_phase_kernels(ga_dev_heap dh, cudaStream_t s, const uint32_t* sizes, uint32_t R, uint32_t T, uint32_t D,
+                              uint32_t round, uint32_t phase, uint64_t* held, ga_log_rec* log, uint64_t* counts,
+                              uint32_t flags, uint32_t block, uint32_t scope) {
+    if (D == 1) {
+        if (scope == 1)
+            k_churn_round<GaBlockPolicy, MAXB><<<nblocks(T, block), block, 0, s>>>(GaBlockPolicy{dh}, sizes, R, T, round, held, log, counts, flags);
+        else if (scope > 1)
+            return launch_cluster(k_churn_round<GaClusterPolicy, MAXB>, nblocks(T, block), block, scope, s, GaClusterPolicy{dh},
+                                  sizes, R, T, round, held, log, counts, flags);
+        else k_churn_round<GaPolicy, MAXB><<<nblocks(T, block), block, 0, s>>>(GaPolicy{dh}, sizes, R, T, round, held, log, counts, flags);
+    } else {
+        if (scope == 1)
+            k_phase<GaBlockPolicy, MAXB><<<nblocks(T, block), block, 0, s>>>(GaBlockPolicy{dh}, sizes, T, round, phase, held, log, counts, flags);
+        else if (scope > 1)
+            return launch_cluster(k_phase<GaClusterPolicy, MAXB>, nblocks(T, block), block, scope, s, GaClusterPolicy{dh}, sizes,
+                                  T, round, phase, held, log, counts, flags);
+        else k_phase<GaPolicy, MAXB><<<nblocks(T, block), block, 0, s>>>(GaPolicy{dh}, sizes, T, round, phase, held, log, counts, flags);
+    }
+    return launched();
+}
+
 }  // namespace
 
 extern "C" {
@@ -434,28 +456,15 @@ ga_status ga_trace_phase(ga_heap_t h, ga_stream_t stream, const uint32_t* sizes,
     if (block == 0) block = 256;
     DeviceGuard g(h->device);
     const ga_dev_heap dh{h->ddesc, h->dev.base};
-    GaPolicy al{dh};
     cudaStream_t s = (cudaStream_t)stream;
     if (!(flags & GA_TRACE_LOG)) log = nullptr;
     const uint32_t scope = (flags >> 8) & 0xF;
     if (!scope_ok(scope, block)) return GA_EINVAL;
     if (D == 1 ? round > R : (round >= R || phase > 1)) return GA_EINVAL;
-    if (D == 1) {
-        if (scope == 1)
-            k_churn_round<GaBlockPolicy><<<nblocks(T, block), block, 0, s>>>(GaBlockPolicy{dh}, sizes, R, T, round, held, log, counts, flags);
-        else if (scope > 1)
-            return launch_cluster(k_churn_round<GaClusterPolicy>, nblocks(T, block), block, scope, s, GaClusterPolicy{dh},
-                                  sizes, R, T, round, held, log, counts, flags);
-        else k_churn_round<GaPolicy><<<nblocks(T, block), block, 0, s>>>(al, sizes, R, T, round, held, log, counts, flags);
-    } else {
-        if (scope == 1)
-            k_phase<GaBlockPolicy><<<nblocks(T, block), block, 0, s>>>(GaBlockPolicy{dh}, sizes, T, round, phase, held, log, counts, flags);
-        else if (scope > 1)
-            return launch_cluster(k_phase<GaClusterPolicy>, nblocks(T, block), block, scope, s, GaClusterPolicy{dh}, sizes,
-                                  T, round, phase, held, log, counts, flags);
-        else k_phase<GaPolicy><<<nblocks(T, block), block, 0, s>>>(al, sizes, T, round, phase, held, log, counts, flags);
-    }
-    return launched();
+    // blocks above 256 threads (the paper's 1..1024 sweep) run
+    // an instantiation bounded at 1024 threads (64 registers)
+    if (block > 256) return trace_phase_kernels<1024>(dh, s, sizes, R, T, D, round, phase, held, log, counts, flags, block, scope);
+    return trace_phase_kernels<256>(dh, s, sizes, R, T, D, round, phase, held, log, counts, flags, block, scope);
 }
 
 ga_status ga_trace_timed_scope(ga_heap_t h, ga_stream_t stream, const uint32_t* sizes, uint32_t R, uint32_t T, uint32_t D,
@@ -550,10 +559,12 @@ ga_status ga_cuda_trace_phase(ga_stream_t stream, const uint32_t* sizes, uint32_
     cudaStream_t s = (cudaStream_t)stream;
     if (D == 1) {
         if (round > R) return GA_EINVAL;
-        k_churn_round<CudaPolicy><<<nblocks(T, block), block, 0, s>>>(al, sizes, R, T, round, held, nullptr, counts, flags);
+        if (block > 256) k_churn_round<CudaPolicy, 1024><<<nblocks(T, block), block, 0, s>>>(al, sizes, R, T, round, held, nullptr, counts, flags);
+        else k_churn_round<CudaPolicy><<<nblocks(T, block), block, 0, s>>>(al, sizes, R, T, round, held, nullptr, counts, flags);
     } else {
         if (round >= R || phase > 1) return GA_EINVAL;
-        k_phase<CudaPolicy><<<nblocks(T, block), block, 0, s>>>(al, sizes, T, round, phase, held, nullptr, counts, flags);
+        if (block > 256) k_phase<CudaPolicy, 1024><<<nblocks(T, block), block, 0, s>>>(al, sizes, T, round, phase, held, nullptr, counts, flags);
+        else k_phase<CudaPolicy><<<nblocks(T, block), block, 0, s>>>(al, sizes, T, round, phase, held, nullptr, counts, flags);
     }
     return launched();
 }
