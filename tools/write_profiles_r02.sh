@@ -35,8 +35,10 @@ rows=list(csv.reader(sys.stdin)); h,u,v=rows[0],rows[1],rows[2]
 def b(n):
     x=float(v[h.index(n)]); un=u[h.index(n)]
     return x*{'byte':1,'Kbyte':1e3,'Mbyte':1e6,'Gbyte':1e9}.get(un,1)
-json.dump({'kernel':'k_timed<GaPolicy,$OCC>','workload':'d4_mixed_pressure','dram_bytes_per_launch':b('dram__bytes_read.sum')+b('dram__bytes_write.sum'),
-           'source':'profiles/r02_ncu_d4_k_timed.txt (ncu --set full, one launch)'}, open('profiles/r02_ncu_traffic.json','w'), indent=1)
+json.dump({'kernel':'k_timed<GaPolicy,$OCC>','workload':'d4_mixed_pressure (full bench trace, one launch)',
+           'dram_bytes_read':b('dram__bytes_read.sum'),'dram_bytes_write':b('dram__bytes_write.sum'),
+           'traffic_bytes':b('dram__bytes_read.sum')+b('dram__bytes_write.sum'),
+           'source':'profiles/r02_ncu_d4_k_timed.txt (ncu --set full --clock-control none, dram__bytes_read.sum + dram__bytes_write.sum)'}, open('profiles/r02_ncu_traffic.json','w'), indent=1)
 "
 fi
 ls gpurun_out/coll_ncu_s*_*.csv > /dev/null 2>&1 && python tools/coll_evidence.py profiles/r02_coll_ncu.json
