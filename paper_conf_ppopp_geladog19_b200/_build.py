@@ -51,6 +51,16 @@ def build_variants(force: bool = False) -> dict:
     return out
 
 
+def build_all(force: bool = False) -> None:
+    """libga.so and every variant, concurrently."""
+    from concurrent.futures import ThreadPoolExecutor
+    with ThreadPoolExecutor(2) as ex:
+        a = ex.submit(build, force)
+        b = ex.submit(build_variants, force)
+        a.result()
+        b.result()
+
+
 def build(force: bool = False, verbose: bool = False, defines=(), out: str | None = None) -> str:
     """Compile libga.so if missing or older than its sources; returns its path.
     `defines` / `out` build a tuning variant (e.g. ("GA_LVL_HINT=1",)) elsewhere."""
@@ -58,16 +68,35 @@ def build(force: bool = False, verbose: bool = False, defines=(), out: str | Non
     if not force and not defines and out is None and not _stale():
         return LIB
     nvcc = os.environ.get("NVCC", "nvcc")
-    cmd = [nvcc, *NVCC_FLAGS, *[f"-D{d}" for d in defines], "-I", INCLUDE, "-I", CSRC,
-           *[os.path.join(CSRC, f) for f in SOURCES], "-o", target + ".tmp"]
+    # one nvcc per translation unit, in parallel (each TU carries its own copy
+    # of the allocator's device code), then one shared-library link
+    flags = [f for f in NVCC_FLAGS if f != "-shared"]
+    common = [*flags, *[f"-D{d}" for d in defines], "-I", INCLUDE, "-I", CSRC]
     if verbose:
-        cmd[1:1] = ["-Xptxas", "-v"]
-    r = subprocess.run(cmd, capture_output=True, text=True)
+        common = ["-Xptxas", "-v", *common]
+    objs = [f"{target}.{os.path.splitext(f)[0]}.o" for f in SOURCES]
+
+    def compile_one(src_obj):
+        src, obj = src_obj
+        return subprocess.run([nvcc, *common, "-c", os.path.join(CSRC, src), "-o", obj], capture_output=True, text=True)
+
+    from concurrent.futures import ThreadPoolExecutor
+    with ThreadPoolExecutor(len(SOURCES)) as ex:
+        results = list(ex.map(compile_one, zip(SOURCES, objs)))
+    for r in results:
+        if r.returncode != 0:
+            sys.stderr.write(r.stdout + r.stderr)
+            raise RuntimeError("nvcc failed building libga.so")
+        if verbose:
+            sys.stderr.write(r.stderr)
+    r = subprocess.run([nvcc, "-gencode", "arch=compute_100a,code=sm_100a", "-shared", "-Xcompiler", "-fPIC",
+                        *objs, "-o", target + ".tmp"], capture_output=True, text=True)
+    for o in objs:
+        if os.path.exists(o):
+            os.remove(o)
     if r.returncode != 0:
         sys.stderr.write(r.stdout + r.stderr)
-        raise RuntimeError("nvcc failed building libga.so")
-    if verbose:
-        sys.stderr.write(r.stderr)
+        raise RuntimeError("nvcc failed linking libga.so")
     os.replace(target + ".tmp", target)
     return target
 
