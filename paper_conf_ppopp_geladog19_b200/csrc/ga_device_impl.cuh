@@ -80,6 +80,9 @@ constexpr int kMaxLevels = 48;
 #ifndef GA_TREE_SPIN_CAP
 #define GA_TREE_SPIN_CAP 256     // max __nanosleep backoff (ns) of a blocked TBuddy wait
 #endif
+#ifndef GA_EAGER_AT
+#define GA_EAGER_AT 9            // empty spans go back to TBuddy at once above GA_EAGER_AT/10 of the heap reserved (10: never)
+#endif
 #ifndef GA_DEFER_RECHECK
 #define GA_DEFER_RECHECK 0       // 1: the lockstep claim validates its slots' page kinds once after the loop, not per iteration
 #endif
@@ -2124,7 +2127,13 @@ static __device__ __forceinline__ void free_body(const ga_desc* h, uint64_t off,
 #pragma unroll
             for (int i = 0; i < 4; i++) if (i < words_of(c) && (ww[i] & valid_mask(c, i))) empty = false;
             if (empty) {
-                if (GA_SPAN_EAGER && is_span(c)) eager = true;   // reclaim after the signal below
+                // reclaim after the signal below: always (GA_SPAN_EAGER), or
+                // once the heap is nearly all reserved (deferred reclamation
+                // keeps empty spans -- whole chunks -- with their arena until a
+                // grower or waiter drains them: the d4 fragmentation excess,
+                // and failed calls at the exhaust level)
+                if (is_span(c) && (GA_SPAN_EAGER || ld_rlx(&h->stats[kStatReserved]) * 10 > h->pages * GA_EAGER_AT))
+                    eager = true;
                 else mark_candidate(h, p, A);
             }
         }
