@@ -80,6 +80,9 @@ constexpr int kMaxLevels = 48;
 #ifndef GA_TREE_SPIN_CAP
 #define GA_TREE_SPIN_CAP 256     // max __nanosleep backoff (ns) of a blocked TBuddy wait
 #endif
+#ifndef GA_SPAN_CLEAR_CHECK
+#define GA_SPAN_CLEAR_CHECK 1    // 1: a failed span claim clears the summary bit only when it is stale
+#endif
 #ifndef GA_EAGER_AT
 #define GA_EAGER_AT 9            // empty spans go back to TBuddy at once above GA_EAGER_AT/10 of the heap reserved (10: never)
 #endif
@@ -1909,9 +1912,17 @@ static __device__ __forceinline__ uint64_t malloc_lockstep(const ga_desc* h, uns
         int wi = 0;
         if (need && (int)lane == pl) {
             got = bin_claim_page(h, page, A, c, __popc(pg), &wi, rot >> 8, !GA_DEFER_RECHECK);
-            if (!got && is_span(c))                            // a full or stale span: drop its summary bit
-                hb3_clear_owned(h, arena_hb(h, A, kAhbNfc + c), page >> kChunkShift, A,
-                                nonfull_word(h, page >> kChunkShift, c), 0);
+            if (!got && is_span(c)) {                          // a full or stale span: drop its summary bit
+                // A full span was already dropped by the claim (nonfull_clear_if_full);
+                // only a STALE summary bit (the chunk's non-full word already
+                // empty, or the chunk no longer A's) needs the clear-then-recheck.
+                const uint64_t ch = page >> kChunkShift;
+                HB3 nb = arena_hb(h, A, kAhbNfc + c);
+                if (!GA_SPAN_CLEAR_CHECK ||
+                    ((ld_rlx(&nb.w0[ch >> 6]) >> (ch & 63)) & 1 &&
+                     (ld_rlx(nonfull_word(h, ch, c)) == 0 || ld_rlx32(&h->chunk_owner[ch]) != A + 1)))
+                    hb3_clear_owned(h, nb, ch, A, nonfull_word(h, ch, c), 0);
+            }
         }
         got = __shfl_sync(bl, got, pl);
         wi = __shfl_sync(bl, wi, pl);
